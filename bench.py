@@ -1,0 +1,405 @@
+#!/usr/bin/env python
+"""bench.py — FP64 GStencils/s of the csx hot path (ConvStencil on B200), one JSON line.
+
+A "step" is one csx_run over one configuration: T base time steps of the stencil on the whole
+grid (every §8(a) row: fused TC passes, remainder pass, FIXED band fix-up).  GStencils/s follows
+Eq 16 (PAPER.md P.1896-1910): T * prod(N) / t / 1e9 with T in base steps (reading A5).
+
+  python bench.py                          # N=1, Box-2D9P 10240^2, T=100 (BASELINE configs[1])
+  torchrun --nproc-per-node N bench.py --gpus N   # weak-scaled slabs: (10240*N) x 10240 (config C5)
+  python bench.py --impl reference         # the CPU oracle on the host cores (bounded sample)
+  python bench.py --config box2d49p --engine direct ...
+
+Timing: W untimed warm-up steps; K timed steps between barrier + cudaDeviceSynchronize, CUDA
+events on the launching stream, max over ranks.  Inputs (839 MB per grid) are larger than the
+126 MB L2, so no explicit flush is needed.  The dominant kernel's time is measured live by the
+library's event hooks (csx_profile_*).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+CONFIGS = {
+    # name: (shape, extents, T, bc, fuse_steps)   — BASELINE.json configs
+    "heat1d_1024": ("heat1d", (1024,), 16, "fixed", 0),                  # C1 (parity config)
+    "box2d9p_10240": ("box2d9p", (10240, 10240), 100, "fixed", 0),       # C2 (headline)
+    "star2d13p_10240": ("star2d13p", (10240, 10240), 100, "fixed", 0),   # C3
+    "box2d49p_10240": ("box2d49p", (10240, 10240), 100, "fixed", 0),     # C3
+    "heat3d_512": ("heat3d", (512, 512, 512), 50, "fixed", 0),           # C4
+    "box3d27p_512": ("box3d27p", (512, 512, 512), 50, "fixed", 0),       # C4
+    "heat1d_10240000": ("heat1d", (10240000,), 1000, "fixed", 0),        # extra (north-star list)
+    "1d5p_10240000": ("1d5p", (10240000,), 1000, "fixed", 0),
+    "heat2d_10240": ("heat2d", (10240, 10240), 100, "fixed", 0),
+}
+DEFAULT = "box2d9p_10240"
+METRIC = "FP64 GStencils/s"
+UNIT = "GStencils/s"
+
+
+def load_json(path):
+    try:
+        with open(path) as f:
+            return json.load(f)
+    except Exception:
+        return None
+
+
+def peaks():
+    mp = load_json(os.path.join(ROOT, "MEASURED_PEAKS.json")) or {}
+    fp = load_json(os.path.join(ROOT, "PEAKS_FP64.json")) or {}
+    hbm = mp.get("hbm_gbs")
+    hbm_src = "MEASURED_PEAKS.json hbm_gbs (measured copy)"
+    if hbm is None:
+        hbm, hbm_src = 6650.0, "fallback 6.65 TB/s (B200_PROFILING.md)"
+    dmma = fp.get("dmma_tflops_sustained") or fp.get("dmma_tflops")
+    dmma_src = "PEAKS_FP64.json dmma_tflops_sustained (on-box DMMA.8x8x4 microbenchmark, peaks/fp64_peaks.cu)"
+    if dmma is None:
+        dmma, dmma_src = 37.2, "nominal 148 SMs x 4 x 512 flop / 16 cyc x 1.965 GHz (no measurement found)"
+    return float(hbm), hbm_src, float(dmma), dmma_src
+
+
+class ClockSampler:
+    """nvidia-smi clocks and throttle reasons sampled every 200 ms during the timed region."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.gpu = gpu_index
+        self.proc = None
+        self.tmp = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=self.tmp, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *exc):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        self.tmp.flush()
+        rows = []
+        try:
+            with open(self.tmp.name) as f:
+                for line in f:
+                    parts = [x.strip() for x in line.split(",")]
+                    if len(parts) >= 9 and parts[1].replace(".", "").isdigit():
+                        rows.append(parts)
+        except Exception:
+            pass
+        finally:
+            try:
+                os.unlink(self.tmp.name)
+            except Exception:
+                pass
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
+        sm = [float(r[1]) for r in rows]
+        smax = max(float(r[2]) for r in rows)
+        loaded = [s for s, r in zip(sm, rows) if float(r[3]) > 250.0] or sm
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({n for r in rows for n, v in zip(names, r[5:9]) if v.lower() == "active"})
+        return {"sm_mhz": statistics.median(loaded), "sm_max_mhz": smax, "reasons": reasons,
+                "samples": len(rows)}
+
+
+def algorithmic_mma(ndim, nk, engine, points, tc_planes):
+    """DMMA.8x8x4 per pass over `points` outputs: Eq 13 generalised by
+    reading A7 (N fragments) and 3D planes for TC_S2R; 4x2/2x4 blocks for TC_TILE."""
+    if engine == "tc_s2r":
+        sw = nk + 1
+        nf = (sw + 7) // 8
+        k = nk if ndim == 1 else nk * nk
+        return points / (8 * sw) * 2 * math.ceil(k / 4) * nf * tc_planes
+    if engine == "tc_tile":
+        a, b = (2, 4) if nk == 5 else (4, 2)
+        kc = 4 * math.ceil((b + nk - 1) / 4)
+        return points / 64 * ((a + nk - 1) * kc // 4) * tc_planes
+    return 0.0
+
+
+def tc_planes_of(name, w):
+    s = synth.SHAPES[name]
+    if s.ndim != 3:
+        return 1
+    return sum(int(np.count_nonzero(w[z]) > 1) for z in range(w.shape[0]))
+
+
+def cpu_oracle_sample(shape, ext, T, bc, w, budget_s=12.0, rows=None):
+    """Time the oracle (as it stands) on the host cores: the full grid of this config (or a
+    slab of it) for as many base steps as fit in ~budget_s."""
+    import oracle
+    cores = len(os.sched_getaffinity(0))
+    u0 = synth.grid(ext, rows=rows)
+    _, s1 = oracle.run(u0, w, bc, 1, nthreads=cores, return_seconds=True)
+    steps = int(max(1, min(T, budget_s / max(s1, 1e-6))))
+    _, secs = oracle.run(u0, w, bc, steps, nthreads=cores, return_seconds=True)
+    pts = u0.size
+    return {"value": steps * pts / secs / 1e9, "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": f"{shape} {'x'.join(map(str, u0.shape))}, {bc}, {steps} of T={T} base steps "
+                      f"(plain-C oracle, OpenMP {cores} threads, {secs:.1f} s)"}
+
+
+def run_reference(args, cfg_name):
+    shape, ext, T, bc, _ = CONFIGS[cfg_name]
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    w = synth.physical_weights(shape)
+    nranks = args.gpus
+    if nranks > 1:
+        ext = (ext[0] * nranks,) + tuple(ext[1:])
+    budget = 8.0
+    t_steps = []
+    cb = None
+    for i in range(args.warmup + args.steps):
+        cb = cpu_oracle_sample(shape, ext, T, bc, w, budget_s=budget)
+        if i >= args.warmup:
+            t_steps.append(cb["value"])
+    value = statistics.median(t_steps) if t_steps else cb["value"]
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": None, "higher_is_better": True, "scaling": "weak" if nranks > 1 else None,
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic (splitmix64 seed 20240302)",
+            "config": {"workload": cfg_name, "grid": list(ext), "T": T, "bc": bc,
+                       "parallelism": "oracle, host cores"},
+            "cpu_baseline": {"kind": "oracle", "cores": cb["cores"], "sample": cb["sample"], "value": value,
+                             "unit": UNIT},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="csx", choices=["csx", "reference"])
+    ap.add_argument("--config", default=DEFAULT, choices=sorted(CONFIGS))
+    ap.add_argument("--engine", default="auto", choices=["auto", "tc_s2r", "tc_tile", "direct"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-comparator", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3  # timing rule: W >= 3
+
+    if args.impl == "reference":
+        run_reference(args, args.config)
+        return
+
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ppopp_chenlwbwmyzcy24_b200 as csx
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    shape, ext, T, bc, tf = CONFIGS[args.config]
+    s = synth.SHAPES[shape]
+    w = synth.physical_weights(shape)
+    gext = (ext[0] * world,) + tuple(ext[1:])  # weak scaling: ext per GPU
+    plan = csx.Plan(gext, w, shape=s.kind, bc=bc, fuse_steps=tf, engine=args.engine)
+    info = plan.info()
+    engine = info["engine_name"]
+    stream = torch.cuda.current_stream()
+    comm = None
+    if world > 1:
+        uid = [csx.csx_nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
+        comm = csx.csx_comm_create(uid[0], rank, world)
+        lo, hi = plan.shard_rows(rank, world)
+        u0 = synth.grid(gext, rows=(lo, hi))
+    else:
+        u0 = synth.grid(gext)
+    d_in = torch.from_numpy(u0).cuda()
+    d_out = torch.empty_like(d_in)
+    n_local = u0.size
+
+    def step():
+        if comm is None:
+            plan.run(d_in, d_out, T, stream)
+        else:
+            plan.run_sharded(comm, d_in, d_out, T, n_local, stream)
+
+    def barrier_sync():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    for _ in range(args.warmup):
+        step()
+    barrier_sync()
+    csx.csx_profile_enable(plan.handle, True)
+    csx.csx_profile_read(plan.handle, reset=True)
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        barrier_sync()
+        ev0.record(stream)
+        for _ in range(args.steps):
+            step()
+        ev1.record(stream)
+        barrier_sync()
+    ms_total = ev0.elapsed_time(ev1)
+    tc_ms, tc_launches, launches = csx.csx_profile_read(plan.handle, reset=True)
+    csx.csx_profile_enable(plan.handle, False)
+    if world > 1:
+        t = torch.tensor([ms_total], device="cuda", dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_total = float(t.item())
+    ms_step = ms_total / args.steps
+    points = int(np.prod(gext))
+    value = T * points / (ms_step * 1e-3) / 1e9
+
+    # ---- roofline of the dominant kernel (the main-pass TC kernel) ----
+    hbm, hbm_src, dmma, dmma_src = peaks()
+    nk, tfm = info["nk"], info["fuse_steps"]
+    local_points = n_local
+    tcp = tc_planes_of(shape, w)
+    roof = None
+    if tc_launches > 0 and engine in ("tc_s2r", "tc_tile"):
+        avg_s = tc_ms / tc_launches * 1e-3
+        mma = algorithmic_mma(s.ndim, nk, engine, local_points, tcp)
+        flops = 512.0 * mma
+        byts = 16.0 * local_points
+        tc_bound = (flops / (dmma * 1e12)) >= (byts / (hbm * 1e9))
+        traffic = None
+        tr = load_json(os.path.join(ROOT, "profiles", "traffic.json")) or {}
+        key = f"{args.config}:{engine}"
+        if key in tr:
+            traffic = tr[key]
+        if tc_bound:
+            achieved = flops / avg_s / 1e12
+            roof = {"bound": "tensor", "achieved": achieved, "peak": dmma, "unit": "TFLOP/s",
+                    "frac": achieved / dmma, "traffic": traffic, "peak_source": dmma_src,
+                    "kernel": f"k_{engine}{s.ndim}d<{nk}>", "avg_launch_ms": avg_s * 1e3,
+                    "launches": tc_launches,
+                    "per_launch": f"{mma:.0f} DMMA.8x8x4 x 512 flop (Eq 13)",
+                    "hbm_frac": byts / avg_s / 1e9 / hbm}
+        else:
+            achieved = byts / avg_s / 1e9
+            roof = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                    "frac": achieved / hbm, "traffic": traffic, "peak_source": hbm_src,
+                    "kernel": f"k_{engine}{s.ndim}d<{nk}>", "avg_launch_ms": avg_s * 1e3,
+                    "launches": tc_launches,
+                    "per_launch": f"16 B x {local_points} points (1 read + 1 write per pass)",
+                    "tensor_frac": flops / avg_s / 1e12 / dmma}
+        roof["tc_share_of_step"] = tc_ms / ms_total if ms_total > 0 else None
+
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic (splitmix64 seed 20240302, dyadic physical weights)",
+            "config": {"workload": args.config, "grid": list(gext), "T": T, "bc": bc,
+                       "fuse_steps": tfm, "nk": nk, "engine": engine,
+                       "parallelism": f"slab{world}" if world > 1 else "single",
+                       "l2": "inputs larger than L2 (839 MB per grid vs 126 MB); no flush needed"},
+            "gpu_launches": int(launches), "roofline": roof}
+
+    # ---- rank-0 extras: clocks, comparator, e2e, cpu baseline ----
+    clocks = clk.summary()
+    line["clocks"] = clocks
+    if rank == 0 and world == 1 and not args.no_comparator and engine != "direct":
+        try:
+            plan.set_engine("direct")
+            plan.run(d_in, d_out, T, stream)
+            torch.cuda.synchronize()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            plan.run(d_in, d_out, T, stream)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            cms = e0.elapsed_time(e1)
+            useful = 2.0 * s.points
+            line["comparator"] = {"engine": "direct (CUDA-core DFMA, temporal blocking)",
+                                  "value": T * points / (cms * 1e-3) / 1e9, "unit": UNIT,
+                                  "useful_flops_per_point_step": useful}
+            plan.set_engine(args.engine)
+        except Exception as e:  # report, do not hide
+            line["comparator"] = {"error": str(e)}
+    if not args.no_e2e:
+        # end to end through the public host-buffer API: pinned host in, H2D, run, D2H
+        if world == 1:
+            h_in = torch.from_numpy(u0).pin_memory().numpy()
+            h_out = torch.empty(u0.shape, dtype=torch.float64).pin_memory().numpy()
+            plan.run_host(h_in, T, h_out, stream)
+            e_steps = max(1, min(args.steps, 3))
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize()
+            e0.record(stream)
+            for _ in range(e_steps):
+                plan.run_host(h_in, T, h_out, stream)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            ems = e0.elapsed_time(e1) / e_steps
+            line["e2e"] = {"value": T * points / (ems * 1e-3) / 1e9, "unit": UNIT,
+                           "h2d_bytes_per_step": int(u0.nbytes), "d2h_bytes_per_step": int(u0.nbytes),
+                           "api": "csx_run_host (pinned host buffers)", "ms_per_step": ems}
+        else:
+            h_in = torch.from_numpy(u0).pin_memory()
+            h_out = torch.empty(u0.shape, dtype=torch.float64).pin_memory()
+            barrier_sync()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            d_in.copy_(h_in, non_blocking=True)
+            step()
+            h_out.copy_(d_out, non_blocking=True)
+            e1.record(stream)
+            barrier_sync()
+            ems = torch.tensor([e0.elapsed_time(e1)], device="cuda", dtype=torch.float64)
+            dist.all_reduce(ems, op=dist.ReduceOp.MAX)
+            ems = float(ems.item())
+            line["e2e"] = {"value": T * points / (ems * 1e-3) / 1e9, "unit": UNIT,
+                           "h2d_bytes_per_step": int(u0.nbytes), "d2h_bytes_per_step": int(u0.nbytes),
+                           "api": "torch pinned copies + csx_run_sharded", "ms_per_step": ems}
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_oracle_sample(shape, gext, T, bc, w)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if comm is not None:
+        csx.csx_comm_destroy(comm)
+    plan.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,177 @@
+/* csx.h — C-ABI of the B200-native ConvStencil hot path (libcsx.so).
+ *
+ * The operation: explicit FP64 stencil time stepping (PAPER.md P.146-149 §1, P.277-287 §2.1):
+ *     u_{t+1}[p] = sum_{o in {-r..r}^d} w[o] * u_t[p + o]
+ * computed as matrix multiplication on FP64 tensor cores (DMMA.8x8x4) by ConvStencil's
+ * stencil2row layout (Eq 5/6, P.731-785), dual tessellation (P.900-959, P.1304-1336), lookup
+ * table + dirty-bits padding (P.1711-1773) and kernel fusion (P.1466-1482).
+ *
+ * Conventions shared by every entry point
+ *   - extents[0] is the SLOWEST axis (C / torch order); grids are dense row-major float64.
+ *   - weights: dense (2r+1)^ndim doubles, row-major over offsets -r..r on every axis; entry
+ *     [i0][i1]... multiplies u[p0 + i0 - r][p1 + i1 - r]... (correlation; the output sits at the
+ *     window centre — Fig 3 and P.1326-1330; readings A2/A3).  STAR shapes must have
+ *     zeros off the axes.
+ *   - Boundary (paper silent, reading A1): CSX_BC_FIXED holds every point within r of
+ *     a face at its initial value; CSX_BC_PERIODIC wraps.
+ *   - timesteps count BASE steps (Eq 16's T, reading A5).
+ *   - All device pointers are plain CUDA device pointers on the current device; the caller
+ *     owns them.  Streams are cudaStream_t passed as void* (NULL = legacy default stream).
+ *
+ * Errors: every function returns csx_status.  Argument checks are synchronous
+ * (CSX_ERR_INVALID_ARGUMENT / CSX_ERR_UNSUPPORTED); launch failures return CSX_ERR_CUDA with
+ * detail in csx_last_error() (thread-local); asynchronous device faults surface at the
+ * caller's next synchronisation.  No function falls back to the CPU.
+ */
+#ifndef CSX_H_
+#define CSX_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  CSX_OK = 0,
+  CSX_ERR_INVALID_ARGUMENT = 1,
+  CSX_ERR_UNSUPPORTED = 2,
+  CSX_ERR_OUT_OF_MEMORY = 3,
+  CSX_ERR_CUDA = 4,
+  CSX_ERR_NCCL = 5,
+  CSX_ERR_INTERNAL = 6
+} csx_status;
+
+/* Stencil shapes, P.277-287: star = axial neighbours only, box = full (2r+1)^d cube. */
+typedef enum { CSX_SHAPE_STAR = 0, CSX_SHAPE_BOX = 1 } csx_shape;
+
+typedef enum { CSX_BC_FIXED = 0, CSX_BC_PERIODIC = 1 } csx_boundary;
+
+/* Which engine runs the fused passes.
+ *   TC_S2R : the paper's design — implicit stencil2row in shared memory through the lookup
+ *            table with dirty-bits padding, dual tessellation 8 x (nk+1) per DMMA chain.
+ *   TC_TILE: B200 variant of the same stencil-as-GEMM on DMMA: 4x2 output blocks per MMA
+ *            column group, A fragments read straight from the staged input tile.
+ *   DIRECT : CUDA-core direct weighted sum with temporal blocking (the comparator, N2).
+ *   AUTO   : TC_TILE where supported, else TC_S2R. */
+typedef enum {
+  CSX_ENGINE_AUTO = 0,
+  CSX_ENGINE_TC_S2R = 1,
+  CSX_ENGINE_TC_TILE = 2,
+  CSX_ENGINE_DIRECT = 3
+} csx_engine;
+
+typedef struct csx_plan_s* csx_plan_t;
+typedef struct csx_comm_s* csx_comm_t;
+
+/* Build a plan (host-only work: fusion depth, composed weights W^(Tf) (P.1466-1482), weight
+ * matrices W_A/W_B (P.961-975), the lookup table (P.1711-1721) and tile geometry).  Device
+ * buffers (weight fragments, LUT, two padded ping-pong grids) are allocated and uploaded at
+ * the first csx_run on the then-current device.
+ *   ndim 1..3; extents[ndim] >= 2*r*Tf+1 each; radius 1..3; fuse_steps 0 = automatic
+ *   (DESIGN.md "Fusion depth"), else Tf >= 1.  *out receives the plan (caller frees with
+ *   csx_plan_destroy).  Errors: INVALID_ARGUMENT (null pointers, bad ndim/radius/extents,
+ *   off-axis star weights, non-finite weights), UNSUPPORTED (a combination no engine covers). */
+csx_status csx_plan(int ndim, const int64_t* extents, csx_shape shape, int radius,
+                    const double* weights, csx_boundary bc, int fuse_steps, csx_plan_t* out);
+
+/* Select the engine for subsequent runs (default AUTO).  UNSUPPORTED if the engine cannot run
+ * this plan's (ndim, radius, Tf). */
+csx_status csx_plan_set_engine(csx_plan_t plan, csx_engine engine);
+
+/* Advance d_in by `timesteps` base steps into d_out (both prod(extents) doubles, device,
+ * 8-byte aligned; d_in == d_out allowed, any other overlap is INVALID_ARGUMENT; d_in is never
+ * written).  Enqueues floor(T/Tf) fused passes plus a remainder pass on `stream` with no host
+ * synchronisation; T == 0 copies.  The plan owns one set of scratch buffers, so a plan must not
+ * be run on two streams concurrently. */
+csx_status csx_run(csx_plan_t plan, const double* d_in, double* d_out, int64_t timesteps,
+                   void* stream);
+
+/* Same as csx_run, but d_in / d_out are HOST buffers (pageable or pinned): copies in, runs,
+ * copies out, synchronises `stream` before returning.  The end-to-end call used by bench.py's
+ * e2e leg. */
+csx_status csx_run_host(csx_plan_t plan, const double* h_in, double* h_out, int64_t timesteps,
+                        void* stream);
+
+/* Multi-GPU (one process per GPU).  nccl_unique_id points to an ncclUniqueId
+ * (NCCL_UNIQUE_ID_BYTES = 128 bytes) created by rank 0 and broadcast by the caller. */
+csx_status csx_comm_create(const void* nccl_unique_id, int rank, int nranks, csx_comm_t* out);
+csx_status csx_comm_destroy(csx_comm_t comm);
+
+/* ncclGetUniqueId into out128 (128 bytes), for rank 0 to broadcast. */
+csx_status csx_nccl_unique_id(void* out128);
+
+/* Rows [lo, hi) of the slowest axis owned by `rank`: lo = floor(rank*N0/nranks). */
+csx_status csx_shard_rows(const csx_plan_t plan, int rank, int nranks, int64_t* lo, int64_t* hi);
+
+/* Slab-sharded run: the plan describes the GLOBAL grid; d_in_local / d_out_local hold this
+ * rank's rows [lo, hi) (csx_shard_rows) x the other extents.  Halos of depth r*Tf are exchanged
+ * with NCCL send/recv every pass (ring for PERIODIC).  Every rank must call with equal plan
+ * parameters and T.  UNSUPPORTED if a rank owns fewer than r*Tf rows. */
+csx_status csx_run_sharded(csx_plan_t plan, csx_comm_t comm, const double* d_in_local,
+                           double* d_out_local, int64_t timesteps, void* stream);
+
+csx_status csx_plan_destroy(csx_plan_t plan);
+
+const char* csx_status_string(csx_status s);
+const char* csx_last_error(void);
+
+/* ----- Introspection (host-only, valid without a GPU) --------------------------------- */
+
+typedef struct {
+  int ndim;
+  int radius;
+  int fuse_steps;        /* Tf of the main passes */
+  int nk;                /* composed window edge 2*r*Tf + 1 */
+  int remainder_steps;   /* reserved (per-run remainder is T mod Tf) */
+  int engine;            /* csx_engine actually used by csx_run */
+  int tile_m, tile_n;    /* CTA output tile (rows x cols of the two fastest axes) */
+  int s2r_pitch;         /* stencil2row smem pitch in doubles (P.1736-1757) */
+  int64_t mma_per_pass;  /* DMMA.8x8x4 instructions one main pass executes (Eq 13, A7) */
+  double tc_flops_per_point_step;  /* 512 * mma_per_pass / (points * Tf) */
+  double useful_flops_per_point_step; /* 2 * nnz(w) */
+} csx_plan_info_t;
+
+csx_status csx_plan_info(const csx_plan_t plan, csx_plan_info_t* info);
+
+/* ----- Measurement hooks (bench.py) -----------------------------------------------------
+ * With profiling enabled, every TC pass kernel launch (the dominant kernel) is bracketed by
+ * CUDA events recorded on the launching stream, and every kernel the library launches is
+ * counted.  csx_profile_read synchronises on the recorded events and returns the summed TC
+ * kernel time (ms) and launch counts since the last reset. */
+csx_status csx_profile_enable(csx_plan_t plan, int enable);
+csx_status csx_profile_read(csx_plan_t plan, double* tc_kernel_ms, int64_t* tc_launches,
+                            int64_t* total_launches, int reset);
+
+/* Composed weights W^(Tf) = w * w * ... (Tf-fold discrete convolution of the offset-indexed
+ * arrays), shape (2*r*Tf+1)^ndim; applying w Tf times equals applying W^(Tf) once on a torus
+ * (Fig 4, P.1466-1482). */
+csx_status csx_compose_weights(int ndim, int radius, const double* weights, int fuse_steps,
+                               double* out);
+
+/* The paper's weight matrices (P.961-975, Fig 3) for an nk x nk window w (row-major):
+ *   W_A[nk*i + j][c] = w[i][j-c] for j >= c, else 0;  W_B[nk*i + j][c] = w[i][j+nk-c] for j < c.
+ * Written as (nk*nk) x (nk+1) row-major arrays.  For 1D pass ndim1 = 1 and an nk-vector. */
+csx_status csx_weight_matrices(int nk, int ndim1, const double* w, double* wa, double* wb);
+
+/* Eq 5 / Eq 6: where input element (x, y) of an m x n grid lands in stencil2row matrix A
+ * (which = 0) or B (which = 1).  Returns 1 and (*row, *col) if it lands, 0 if the element is
+ * not part of that matrix (it is then a "dirty bit", P.1759-1773). */
+int csx_stencil2row_index(int nk, int which, int64_t x, int64_t y, int64_t* row, int64_t* col);
+
+/* Shared-memory conflict degree of one FP64 m8n8k4 A-fragment load (two 4x4 requests,
+ * P.1736-1757) from a stencil2row tile of pitch `pitch` doubles at column offset `col`:
+ * the max number of distinct 8-byte words one 4-byte bank must serve per request. */
+int csx_fragment_bank_conflicts(int pitch, int col);
+
+/* Copy the plan's lookup table: per element of the CTA input region (row-major,
+ * region_rows x region_cols) the smem offsets in A and B (dirty slots included).  With lut
+ * NULL, only *count is returned. */
+csx_status csx_plan_lut(const csx_plan_t plan, int32_t* lut_a, int32_t* lut_b, int64_t* count,
+                        int* region_rows, int* region_cols);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CSX_H_ */

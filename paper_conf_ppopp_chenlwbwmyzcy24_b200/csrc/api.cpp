@@ -1,0 +1,517 @@
+// api.cpp — the C-ABI of libcsx.so (include/csx.h): argument validation, device state, and
+// the pass loop of csx_run.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "csx_internal.h"
+#include "csx_run.h"
+#include "kernels.cuh"
+
+namespace csx {
+
+static thread_local std::string g_err;
+
+void set_error(const std::string& msg) { g_err = msg; }
+
+csx_status fail(csx_status s, const std::string& msg) {
+  g_err = msg;
+  return s;
+}
+
+csx_status cuda_fail(cudaError_t e, const char* where) {
+  g_err = std::string(where) + ": " + cudaGetErrorString(e);
+  return CSX_ERR_CUDA;
+}
+
+#define CSX_CUDA(call, where)                   \
+  do {                                          \
+    cudaError_t e_ = (call);                    \
+    if (e_ != cudaSuccess) return cuda_fail(e_, where); \
+  } while (0)
+
+// Tile shape of the direct kernel (engine DIRECT and the FIXED band fix-up).
+void direct_tile(int ndim, int* B) {
+  if (ndim == 1) { B[0] = 1; B[1] = 1; B[2] = 1024; }
+  else if (ndim == 2) { B[0] = 1; B[1] = 32; B[2] = 64; }
+  else { B[0] = 8; B[1] = 8; B[2] = 32; }
+}
+
+// Tiles of the direct kernel that intersect the band of width `band` along a GLOBAL face.
+// E = local extents, gorg = local origin in global coordinates, GE = global extents.
+std::vector<int32_t> band_tiles(int ndim, const int64_t* E, const int64_t* gorg, const int64_t* GE,
+                                int band) {
+  int B[3];
+  direct_tile(ndim, B);
+  int64_t nt[3];
+  for (int a = 0; a < 3; ++a) nt[a] = (E[a] + B[a] - 1) / B[a];
+  std::vector<int32_t> out;
+  for (int64_t t0 = 0; t0 < nt[0]; ++t0)
+    for (int64_t t1 = 0; t1 < nt[1]; ++t1)
+      for (int64_t t2 = 0; t2 < nt[2]; ++t2) {
+        const int64_t t[3] = {t0, t1, t2};
+        bool hit = false;
+        for (int a = 3 - ndim; a < 3 && !hit; ++a) {
+          const int64_t lo = gorg[a] + t[a] * B[a];
+          const int64_t hi = std::min(gorg[a] + E[a], lo + B[a]);  // exclusive
+          if (lo < band || hi > GE[a] - band) hit = true;
+        }
+        if (hit) out.push_back((int32_t)((t0 * nt[1] + t1) * nt[2] + t2));
+      }
+  return out;
+}
+
+static csx_status upload_pass(Pass& ps) {
+  if (ps.uploaded) return CSX_OK;
+  if (ps.s2r_ok) {
+    CSX_CUDA(cudaMalloc(&ps.d_frags, ps.frags.size() * sizeof(double)), "cudaMalloc(frags)");
+    CSX_CUDA(cudaMemcpy(ps.d_frags, ps.frags.data(), ps.frags.size() * sizeof(double),
+                        cudaMemcpyHostToDevice), "upload frags");
+    const size_t ne = ps.lut_g.size();
+    std::vector<int32_t> il(2 * ne);
+    for (size_t e = 0; e < ne; ++e) {
+      il[2 * e] = ps.lut_g[e];
+      il[2 * e + 1] = (int32_t)((uint32_t)ps.lut_a[e] | ((uint32_t)ps.lut_b[e] << 16));
+    }
+    CSX_CUDA(cudaMalloc(&ps.d_lut, il.size() * sizeof(int32_t)), "cudaMalloc(lut)");
+    CSX_CUDA(cudaMemcpy(ps.d_lut, il.data(), il.size() * sizeof(int32_t), cudaMemcpyHostToDevice),
+             "upload lut");
+  }
+  if (ps.tile_ok) {
+    CSX_CUDA(cudaMalloc(&ps.d_tile_frags, ps.tile_frags.size() * sizeof(double)), "cudaMalloc");
+    CSX_CUDA(cudaMemcpy(ps.d_tile_frags, ps.tile_frags.data(),
+                        ps.tile_frags.size() * sizeof(double), cudaMemcpyHostToDevice), "upload");
+  }
+  CSX_CUDA(cudaMalloc(&ps.d_wc, ps.wc.size() * sizeof(double)), "cudaMalloc(wc)");
+  CSX_CUDA(cudaMemcpy(ps.d_wc, ps.wc.data(), ps.wc.size() * sizeof(double), cudaMemcpyHostToDevice),
+           "upload wc");
+  ps.uploaded = true;
+  return CSX_OK;
+}
+
+csx_status ensure_device(csx_plan_s* p) {
+  int dev = 0;
+  CSX_CUDA(cudaGetDevice(&dev), "cudaGetDevice");
+  if (p->device >= 0) {
+    if (dev != p->device) return fail(CSX_ERR_INVALID_ARGUMENT, "plan used on another device");
+    return CSX_OK;
+  }
+  for (auto& ps : p->passes) {
+    csx_status s = upload_pass(ps);
+    if (s != CSX_OK) return s;
+  }
+  CSX_CUDA(cudaMalloc(&p->d_wbase, p->w.size() * sizeof(double)), "cudaMalloc(w)");
+  CSX_CUDA(cudaMemcpy(p->d_wbase, p->w.data(), p->w.size() * sizeof(double),
+                      cudaMemcpyHostToDevice), "upload w");
+  p->device = dev;
+  return CSX_OK;
+}
+
+csx_status ensure_grid(csx_plan_s* p, Padded* pd, double** bufs, const int64_t* E) {
+  if (bufs[0]) return CSX_OK;
+  layout_padded(p, E, pd);
+  const size_t bytes = (size_t)pd->elems() * sizeof(double);
+  for (int i = 0; i < 2; ++i) {
+    cudaError_t e = cudaMalloc(&bufs[i], bytes);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      return fail(CSX_ERR_OUT_OF_MEMORY, "cudaMalloc of a padded grid failed");
+    }
+    CSX_CUDA(cudaMemset(bufs[i], 0, bytes), "cudaMemset");
+  }
+  return CSX_OK;
+}
+
+// One fused pass of Tf' steps from the padded source to dst (padded scratch or user output).
+// ctx describes the local grid and its place in the global grid (sharded runs).
+csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) {
+  csx_engine eng = p->engine;
+  cudaError_t e = cudaSuccess;
+  if (eng == CSX_ENGINE_TC_S2R || eng == CSX_ENGINE_TC_TILE) {
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    const bool prof = p->prof && ps.tf == p->tf;  // time the main-pass (dominant) kernel only
+    if (prof) {
+      if (p->prof_used + 2 > p->prof_events.size()) {
+        for (int k = 0; k < 64; ++k) {
+          cudaEvent_t ev;
+          CSX_CUDA(cudaEventCreate(&ev), "cudaEventCreate");
+          p->prof_events.push_back(ev);
+        }
+      }
+      ev0 = (cudaEvent_t)p->prof_events[p->prof_used++];
+      ev1 = (cudaEvent_t)p->prof_events[p->prof_used++];
+      CSX_CUDA(cudaEventRecord(ev0, st), "cudaEventRecord");
+    }
+    S2RArgs a;
+    a.src = c.src;
+    a.dst = c.dst;
+    a.E0 = c.E[0]; a.E1 = c.E[1]; a.E2 = c.E[2];
+    a.lut = reinterpret_cast<const int2*>(ps.d_lut);
+    a.wc = ps.d_wc;
+    if (eng == CSX_ENGINE_TC_TILE) {
+      a.frags = ps.d_tile_frags;
+      e = launch_tile(p->ndim, ps.nk, a, st);
+    } else {
+      a.frags = ps.d_frags;
+      int tc_mask = 0;
+      if (p->ndim == 1) {
+        a.tiles_x = (int)((c.E[2] + ps.bn - 1) / ps.bn);
+        a.tiles_y = 1;
+        a.ntiles = a.tiles_x;
+      } else {
+        a.tiles_x = (int)((c.E[2] + ps.bn - 1) / ps.bn);
+        a.tiles_y = (int)((c.E[1] + ps.bm - 1) / ps.bm);
+        a.ntiles = (int64_t)a.tiles_x * a.tiles_y;
+        if (p->ndim == 3) {
+          const int64_t zchunk = 64;
+          a.ntiles *= (c.E[0] + zchunk - 1) / zchunk;
+          for (int dz = 0; dz < ps.nk; ++dz) tc_mask |= ps.plane_is_tc[dz] << dz;
+        }
+      }
+      e = launch_s2r(p->ndim, ps.nk, ps.nf, a, tc_mask, st);
+    }
+    if (e != cudaSuccess) return cuda_fail(e, "TC pass launch");
+    if (prof) CSX_CUDA(cudaEventRecord(ev1, st), "cudaEventRecord");
+    if (ps.tf == p->tf) p->n_tc_launches += 1;
+    p->n_launches += 1;
+  }
+  const bool direct_all = eng == CSX_ENGINE_DIRECT;
+  if (direct_all || p->bc == CSX_BC_FIXED) {
+    DirectArgs d;
+    d.src = c.src;
+    d.dst = c.dst;
+    for (int a2 = 0; a2 < 3; ++a2) {
+      d.E[a2] = c.E[a2];
+      d.real[a2] = a2 >= 3 - p->ndim;
+      d.gorg[a2] = c.gorg[a2];
+      d.GE[a2] = p->E[a2];
+    }
+    d.r = p->radius;
+    d.tf = ps.tf;
+    d.fixed_bc = p->bc == CSX_BC_FIXED;
+    d.band = direct_all ? 0 : p->radius * ps.tf;
+    direct_tile(p->ndim, d.B);
+    for (int a2 = 0; a2 < 3; ++a2) d.tiles[a2] = (int)((c.E[a2] + d.B[a2] - 1) / d.B[a2]);
+    d.w = p->d_wbase;
+    d.ndim = p->ndim;
+    if (direct_all) {
+      d.tile_list = nullptr;
+      d.ntiles = (int64_t)d.tiles[0] * d.tiles[1] * d.tiles[2];
+    } else {
+      d.tile_list = c.band_tiles;
+      d.ntiles = c.n_band_tiles;
+    }
+    e = launch_direct(d, st);
+    if (e != cudaSuccess) return cuda_fail(e, "direct/fix-up launch");
+    if (d.ntiles > 0) p->n_launches += 1;
+  }
+  return CSX_OK;
+}
+
+}  // namespace csx
+
+using namespace csx;
+
+extern "C" {
+
+const char* csx_status_string(csx_status s) {
+  switch (s) {
+    case CSX_OK: return "CSX_OK";
+    case CSX_ERR_INVALID_ARGUMENT: return "CSX_ERR_INVALID_ARGUMENT";
+    case CSX_ERR_UNSUPPORTED: return "CSX_ERR_UNSUPPORTED";
+    case CSX_ERR_OUT_OF_MEMORY: return "CSX_ERR_OUT_OF_MEMORY";
+    case CSX_ERR_CUDA: return "CSX_ERR_CUDA";
+    case CSX_ERR_NCCL: return "CSX_ERR_NCCL";
+    case CSX_ERR_INTERNAL: return "CSX_ERR_INTERNAL";
+  }
+  return "CSX_ERR_UNKNOWN";
+}
+
+const char* csx_last_error(void) { return g_err.c_str(); }
+
+static bool engine_ok(const csx_plan_s* p, csx_engine e) {
+  for (const auto& ps : p->passes) {
+    if (e == CSX_ENGINE_TC_S2R && !ps.s2r_ok) return false;
+    if (e == CSX_ENGINE_TC_TILE && !(ps.tile_ok && tile_kernel_exists(p->ndim, ps.nk))) return false;
+  }
+  return true;
+}
+
+csx_status csx_plan(int ndim, const int64_t* extents, csx_shape shape, int radius,
+                    const double* weights, csx_boundary bc, int fuse_steps, csx_plan_t* out) {
+  if (!out) return fail(CSX_ERR_INVALID_ARGUMENT, "out is NULL");
+  *out = nullptr;
+  if (!extents || !weights) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL extents or weights");
+  if (ndim < 1 || ndim > 3) return fail(CSX_ERR_INVALID_ARGUMENT, "ndim must be 1, 2 or 3");
+  if (radius < 1 || radius > 3) return fail(CSX_ERR_INVALID_ARGUMENT, "radius must be 1..3");
+  if (shape != CSX_SHAPE_STAR && shape != CSX_SHAPE_BOX)
+    return fail(CSX_ERR_INVALID_ARGUMENT, "unknown shape");
+  if (bc != CSX_BC_FIXED && bc != CSX_BC_PERIODIC)
+    return fail(CSX_ERR_INVALID_ARGUMENT, "unknown boundary");
+  if (fuse_steps < 0 || fuse_steps > 16) return fail(CSX_ERR_INVALID_ARGUMENT, "fuse_steps out of range");
+  csx_plan_s* p = new (std::nothrow) csx_plan_s();
+  if (!p) return fail(CSX_ERR_OUT_OF_MEMORY, "plan allocation");
+  p->ndim = ndim;
+  p->radius = radius;
+  p->shape = shape;
+  p->bc = bc;
+  for (int a = 0; a < ndim; ++a) {
+    if (extents[a] < 1) { delete p; return fail(CSX_ERR_INVALID_ARGUMENT, "extent < 1"); }
+    p->ext[a] = extents[a];
+    p->E[3 - ndim + a] = extents[a];
+  }
+  const int n = 2 * radius + 1;
+  int64_t dense = 1;
+  for (int a = 0; a < ndim; ++a) dense *= n;
+  p->w.assign(weights, weights + dense);
+  for (int64_t i = 0; i < dense; ++i) {
+    if (!std::isfinite(p->w[i])) { delete p; return fail(CSX_ERR_INVALID_ARGUMENT, "non-finite weight"); }
+    if (p->w[i] != 0.0) ++p->nnz;
+    if (shape == CSX_SHAPE_STAR && p->w[i] != 0.0) {
+      int64_t rem = i;
+      int offaxis = 0;
+      for (int a = 0; a < ndim; ++a) { offaxis += (rem % n) != radius; rem /= n; }
+      if (offaxis > 1) { delete p; return fail(CSX_ERR_INVALID_ARGUMENT, "STAR weight off the axes"); }
+    }
+  }
+  p->tf = fuse_steps;
+  csx_status s = build_plan(p);
+  if (s != CSX_OK) { delete p; return s; }
+  p->engine_req = CSX_ENGINE_AUTO;
+  if (engine_ok(p, CSX_ENGINE_TC_TILE)) p->engine = CSX_ENGINE_TC_TILE;
+  else if (engine_ok(p, CSX_ENGINE_TC_S2R)) p->engine = CSX_ENGINE_TC_S2R;
+  else p->engine = CSX_ENGINE_DIRECT;
+  *out = p;
+  return CSX_OK;
+}
+
+csx_status csx_plan_set_engine(csx_plan_t p, csx_engine e) {
+  if (!p) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL plan");
+  if (e == CSX_ENGINE_AUTO) {
+    p->engine_req = e;
+    if (engine_ok(p, CSX_ENGINE_TC_TILE)) p->engine = CSX_ENGINE_TC_TILE;
+    else if (engine_ok(p, CSX_ENGINE_TC_S2R)) p->engine = CSX_ENGINE_TC_S2R;
+    else p->engine = CSX_ENGINE_DIRECT;
+    return CSX_OK;
+  }
+  if (e != CSX_ENGINE_TC_S2R && e != CSX_ENGINE_TC_TILE && e != CSX_ENGINE_DIRECT)
+    return fail(CSX_ERR_INVALID_ARGUMENT, "unknown engine");
+  if (!engine_ok(p, e)) return fail(CSX_ERR_UNSUPPORTED, "engine cannot run this plan");
+  p->engine_req = e;
+  p->engine = e;
+  return CSX_OK;
+}
+
+csx_status csx_run(csx_plan_t p, const double* d_in, double* d_out, int64_t T, void* stream) {
+  if (!p || !d_in || !d_out) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL argument");
+  if (T < 0) return fail(CSX_ERR_INVALID_ARGUMENT, "timesteps < 0");
+  if ((reinterpret_cast<uintptr_t>(d_in) | reinterpret_cast<uintptr_t>(d_out)) & 7)
+    return fail(CSX_ERR_INVALID_ARGUMENT, "grids must be 8-byte aligned");
+  const int64_t n = p->E[0] * p->E[1] * p->E[2];
+  if (d_in != d_out && d_in < d_out + n && d_out < d_in + n)
+    return fail(CSX_ERR_INVALID_ARGUMENT, "d_in and d_out overlap");
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  csx_status s = ensure_device(p);
+  if (s != CSX_OK) return s;
+  if (T == 0) {
+    if (d_in != d_out)
+      CSX_CUDA(cudaMemcpyAsync(d_out, d_in, n * sizeof(double), cudaMemcpyDeviceToDevice, st), "copy");
+    return CSX_OK;
+  }
+  s = ensure_grid(p, &p->pad, p->d_buf, p->E);
+  if (s != CSX_OK) return s;
+  if (p->bc == CSX_BC_FIXED && p->band_tiles_n < 0) {
+    const int64_t zero[3] = {0, 0, 0};
+    std::vector<int32_t> bt = band_tiles(p->ndim, p->E, zero, p->E, p->halo);
+    p->band_tiles_n = (int64_t)bt.size();
+    CSX_CUDA(cudaMalloc(&p->d_band_tiles, std::max<size_t>(1, bt.size()) * sizeof(int32_t)), "cudaMalloc");
+    CSX_CUDA(cudaMemcpy(p->d_band_tiles, bt.data(), bt.size() * sizeof(int32_t), cudaMemcpyHostToDevice),
+             "upload band tiles");
+  }
+  return run_local(p, d_in, d_out, T, st);
+}
+
+csx_status csx_run_host(csx_plan_t p, const double* h_in, double* h_out, int64_t T, void* stream) {
+  if (!p || !h_in || !h_out) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL argument");
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  const int64_t n = p->E[0] * p->E[1] * p->E[2];
+  csx_status s = ensure_device(p);
+  if (s != CSX_OK) return s;
+  if (!p->d_dense) {
+    cudaError_t e = cudaMalloc(&p->d_dense, n * sizeof(double));
+    if (e != cudaSuccess) { cudaGetLastError(); return fail(CSX_ERR_OUT_OF_MEMORY, "cudaMalloc(dense)"); }
+  }
+  CSX_CUDA(cudaMemcpyAsync(p->d_dense, h_in, n * sizeof(double), cudaMemcpyHostToDevice, st), "H2D");
+  s = csx_run(p, p->d_dense, p->d_dense, T, stream);
+  if (s != CSX_OK) return s;
+  CSX_CUDA(cudaMemcpyAsync(h_out, p->d_dense, n * sizeof(double), cudaMemcpyDeviceToHost, st), "D2H");
+  CSX_CUDA(cudaStreamSynchronize(st), "sync");
+  return CSX_OK;
+}
+
+csx_status csx_profile_enable(csx_plan_t p, int enable) {
+  if (!p) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL plan");
+  p->prof = enable != 0;
+  return CSX_OK;
+}
+
+csx_status csx_profile_read(csx_plan_t p, double* tc_ms, int64_t* tc_launches, int64_t* total,
+                            int reset) {
+  if (!p) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL plan");
+  double ms = 0.0;
+  for (size_t i = 0; i + 1 < p->prof_used; i += 2) {
+    cudaEvent_t a = (cudaEvent_t)p->prof_events[i], b = (cudaEvent_t)p->prof_events[i + 1];
+    CSX_CUDA(cudaEventSynchronize(b), "cudaEventSynchronize");
+    float f = 0.f;
+    CSX_CUDA(cudaEventElapsedTime(&f, a, b), "cudaEventElapsedTime");
+    ms += f;
+  }
+  if (tc_ms) *tc_ms = ms;
+  if (tc_launches) *tc_launches = p->n_tc_launches;
+  if (total) *total = p->n_launches;
+  if (reset) {
+    p->prof_used = 0;
+    p->n_tc_launches = 0;
+    p->n_launches = 0;
+  }
+  return CSX_OK;
+}
+
+csx_status csx_plan_destroy(csx_plan_t p) {
+  if (!p) return CSX_OK;
+  for (void* ev : p->prof_events) cudaEventDestroy((cudaEvent_t)ev);
+  if (p->device >= 0) {
+    int cur = 0;
+    cudaGetDevice(&cur);
+    cudaSetDevice(p->device);
+    for (auto& ps : p->passes) {
+      cudaFree(ps.d_frags);
+      cudaFree(ps.d_lut);
+      cudaFree(ps.d_tile_frags);
+      cudaFree(ps.d_wc);
+    }
+    cudaFree(p->d_buf[0]);
+    cudaFree(p->d_buf[1]);
+    cudaFree(p->d_wbase);
+    cudaFree(p->d_dense);
+    cudaFree(p->d_band_tiles);
+    cudaFree(p->d_sbuf[0]);
+    cudaFree(p->d_sbuf[1]);
+    cudaFree(p->d_sband_tiles);
+    cudaSetDevice(cur);
+  }
+  delete p;
+  return CSX_OK;
+}
+
+csx_status csx_plan_info(const csx_plan_t p, csx_plan_info_t* info) {
+  if (!p || !info) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL argument");
+  const Pass& ps = p->passes[p->tf - 1];
+  std::memset(info, 0, sizeof(*info));
+  info->ndim = p->ndim;
+  info->radius = p->radius;
+  info->fuse_steps = p->tf;
+  info->nk = ps.nk;
+  info->engine = p->engine;
+  info->tile_m = ps.bm;
+  info->tile_n = ps.bn;
+  info->s2r_pitch = ps.pitch;
+  info->mma_per_pass = p->engine == CSX_ENGINE_TC_TILE ? ps.tile_mma_per_pass
+                       : p->engine == CSX_ENGINE_TC_S2R ? ps.mma_per_pass : 0;
+  const double pts = (double)(p->E[0] * p->E[1] * p->E[2]);
+  info->tc_flops_per_point_step = 512.0 * (double)info->mma_per_pass / (pts * ps.tf);
+  info->useful_flops_per_point_step = 2.0 * p->nnz;
+  return CSX_OK;
+}
+
+csx_status csx_compose_weights(int ndim, int radius, const double* w, int tf, double* out) {
+  if (!w || !out || ndim < 1 || ndim > 3 || radius < 1 || radius > 7 || tf < 1 || tf > 16)
+    return fail(CSX_ERR_INVALID_ARGUMENT, "bad argument");
+  int64_t dense = 1;
+  for (int a = 0; a < ndim; ++a) dense *= 2 * radius + 1;
+  std::vector<double> base(w, w + dense);
+  std::vector<double> c = compose(ndim, radius, base, tf);
+  std::memcpy(out, c.data(), c.size() * sizeof(double));
+  return CSX_OK;
+}
+
+csx_status csx_weight_matrices(int nk, int ndim1, const double* w, double* wa, double* wb) {
+  if (!w || !wa || !wb || nk < 1 || nk > 31) return fail(CSX_ERR_INVALID_ARGUMENT, "bad argument");
+  weight_matrices(nk, ndim1, w, wa, wb);
+  return CSX_OK;
+}
+
+int csx_stencil2row_index(int nk, int which, int64_t x, int64_t y, int64_t* row, int64_t* col) {
+  if (!row || !col || nk < 1 || x < 0 || y < 0) return 0;
+  return s2r_index(nk, which, x, y, row, col) ? 1 : 0;
+}
+
+int csx_fragment_bank_conflicts(int pitch, int col) { return fragment_conflicts(pitch, col); }
+
+csx_status csx_plan_lut(const csx_plan_t p, int32_t* lut_a, int32_t* lut_b, int64_t* count,
+                        int* region_rows, int* region_cols) {
+  if (!p || !count) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL argument");
+  const Pass& ps = p->passes[p->tf - 1];
+  if (!ps.s2r_ok) return fail(CSX_ERR_UNSUPPORTED, "plan has no stencil2row LUT");
+  *count = (int64_t)ps.lut_a.size();
+  if (region_rows) *region_rows = ps.rr;
+  if (region_cols) *region_cols = ps.rc;
+  if (lut_a) std::memcpy(lut_a, ps.lut_a.data(), ps.lut_a.size() * sizeof(int32_t));
+  if (lut_b) std::memcpy(lut_b, ps.lut_b.data(), ps.lut_b.size() * sizeof(int32_t));
+  return CSX_OK;
+}
+
+}  // extern "C"
+
+namespace csx {
+
+// The pass loop: pack d_in into the padded grid, then floor(T/Tf) fused
+// passes plus one remainder pass of T mod Tf steps, ping-ponging between the two padded
+// grids; the last pass writes straight into d_out.  PERIODIC ghosts are refreshed after every
+// pass; FIXED bands are recomputed by the fix-up inside run_pass.
+csx_status run_local(csx_plan_s* p, const double* d_in, double* d_out, int64_t T, cudaStream_t st) {
+  const Padded& pd = p->pad;
+  const int real[3] = {p->ndim == 3, p->ndim >= 2, 1};
+  View b[2];
+  for (int i = 0; i < 2; ++i) b[i] = View{p->d_buf[i] + pd.origin(), pd.s0, pd.s1};
+  cudaError_t e = launch_pack(d_in, b[0], p->E, st);
+  if (e != cudaSuccess) return cuda_fail(e, "pack");
+  p->n_launches += 1;
+  const int nghost = real[0] + real[1] + real[2];
+  if (p->bc == CSX_BC_PERIODIC) {
+    e = launch_ghost_fill(b[0], p->E, real, real, p->halo, st);
+    if (e != cudaSuccess) return cuda_fail(e, "ghost fill");
+    p->n_launches += nghost;
+  }
+  const int64_t nmain = T / p->tf;
+  const int rem = (int)(T % p->tf);
+  const int64_t npass = nmain + (rem ? 1 : 0);
+  const View out{d_out, p->E[1] * p->E[2], p->E[2]};
+  int cur = 0;
+  for (int64_t i = 0; i < npass; ++i) {
+    const int tfp = i < nmain ? p->tf : rem;
+    const bool last = i == npass - 1;
+    PassCtx c;
+    c.src = CView{b[cur].p, b[cur].s0, b[cur].s1};
+    c.dst = last ? out : b[cur ^ 1];
+    for (int a = 0; a < 3; ++a) { c.E[a] = p->E[a]; c.gorg[a] = 0; }
+    c.band_tiles = p->d_band_tiles;
+    c.n_band_tiles = p->band_tiles_n;
+    csx_status s = run_pass(p, p->passes[tfp - 1], c, st);
+    if (s != CSX_OK) return s;
+    if (!last && p->bc == CSX_BC_PERIODIC) {
+      e = launch_ghost_fill(b[cur ^ 1], p->E, real, real, p->halo, st);
+      if (e != cudaSuccess) return cuda_fail(e, "ghost fill");
+      p->n_launches += nghost;
+    }
+    cur ^= 1;
+  }
+  return CSX_OK;
+}
+
+}  // namespace csx

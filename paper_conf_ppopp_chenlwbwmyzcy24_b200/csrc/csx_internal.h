@@ -1,0 +1,129 @@
+// csx_internal.h — plan representation shared by the host planner (planner.cpp), the C-ABI
+// (api.cpp) and the kernel launchers (*.cu).  Product code only; nothing here is shared with
+// oracle/.
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "../../include/csx.h"
+
+namespace csx {
+
+constexpr int kMaxNK = 15;          // largest composed window edge any engine accepts
+constexpr int kWarp = 32;
+
+// Set the thread-local error detail returned by csx_last_error().
+void set_error(const std::string& msg);
+csx_status fail(csx_status s, const std::string& msg);
+
+// ---- host planning (planner.cpp) -------------------------------------------------------
+
+// W^(Tf): Tf-fold discrete convolution of the offset-indexed (2r+1)^d array (P.1466-1482).
+std::vector<double> compose(int ndim, int radius, const std::vector<double>& w, int tf);
+
+// Paper weight matrices (P.961-975): (nk*nk) x (nk+1) row-major (2D) or nk x (nk+1) (1D).
+void weight_matrices(int nk, int ndim1, const double* w, double* wa, double* wb);
+
+// Eq 5 / Eq 6 mapping.  Returns true if (x, y) lands in matrix `which` (0 = A, 1 = B).
+bool s2r_index(int nk, int which, int64_t x, int64_t y, int64_t* row, int64_t* col);
+
+// Max 8-byte words per 4-byte bank over the two 4x4 requests of one m8n8k4 A fragment
+// read from a stencil2row tile with pitch `pitch` (doubles), fragment column `col`.
+int fragment_conflicts(int pitch, int col);
+
+// Smallest pitch >= min_pitch that is conflict-free for every fragment column (Fig 5).
+int choose_pitch(int min_pitch);
+
+// One fused-pass configuration (a "sub-plan"): Tf' steps, composed window nk = 2 r Tf' + 1.
+struct Pass {
+  int tf = 0;
+  int nk = 0;
+  std::vector<double> wc;          // composed weights, nk^ndim
+  // --- TC_S2R geometry (2D: nk x nk window; 1D: nk; 3D: per-plane 2D windows) ---
+  int sw = 0;                      // strip width nk + 1 (outputs per strip)
+  int ks = 0;                      // k-slices per weight matrix (ceil(K/4))
+  int nf = 0;                      // N fragments ceil((nk+1)/8)
+  int bm = 0, bn = 0;              // CTA output tile (rows, cols)
+  int rr = 0, rc = 0;              // CTA input region rows, cols
+  int pitch = 0;                   // stencil2row smem pitch (doubles)
+  int planes = 1;                  // 3D: number of z offsets (nk); 1D/2D: 1
+  int tc_planes = 1;               // 3D: planes computed on tensor cores
+  std::vector<int> plane_is_tc;    // 3D: per z offset, 1 = TC, 0 = CUDA-core single tap
+  std::vector<double> frags;       // per-lane DMMA B fragments [plane][A|B][nf][ks][32]
+  std::vector<int32_t> lut_g;      // per region element: offset in the padded source grid
+  std::vector<int32_t> lut_a;      // per region element: smem offset in stencil2row A
+  std::vector<int32_t> lut_b;      // per region element: smem offset in stencil2row B
+  int64_t mma_per_pass = 0;        // DMMA instructions per pass over the whole grid
+  // --- TC_TILE geometry ---
+  int tile_ok = 0;
+  bool s2r_ok = false;              // a TC_S2R kernel exists for (ndim, nk)
+  std::vector<double> tile_frags;  // [plane][slice][32] fragments for the 4x2-block GEMM
+  int tile_ks = 0;                 // k-slices per output block (K / 4)
+  int tile_a = 0, tile_b = 0;      // output block a rows x b cols (a * b = 8 = DMMA N)
+  int tile_kc = 0;                 // padded region row length of one block (multiple of 4)
+  int64_t tile_mma_per_pass = 0;
+  // device copies (owned)
+  double* d_frags = nullptr;
+  int32_t* d_lut = nullptr;        // interleaved {g, a | b << 16} pairs
+  double* d_tile_frags = nullptr;
+  double* d_wc = nullptr;          // composed weights on the device (direct / 3D CUDA-core taps)
+  bool uploaded = false;
+};
+
+// A padded ping-pong grid: 3 normalised axes (missing leading axes have extent 1).
+struct Padded {
+  int64_t E[3] = {1, 1, 1};        // interior extents
+  int64_t O[3] = {0, 0, 0};        // interior origin inside the allocation
+  int64_t A[3] = {1, 1, 1};        // allocated extents (A[2] is the row pitch)
+  int64_t s0 = 0, s1 = 0;          // strides of axes 0 and 1 (axis 2 stride is 1)
+  int64_t elems() const { return A[0] * A[1] * A[2]; }
+  int64_t origin() const { return O[0] * s0 + O[1] * s1 + O[2]; }
+};
+
+}  // namespace csx
+
+struct csx_plan_s {
+  int ndim = 0;
+  int64_t ext[3] = {1, 1, 1};      // user extents (ext[0] slowest), ndim of them valid
+  int64_t E[3] = {1, 1, 1};        // normalised to 3 axes
+  int radius = 0;
+  csx_shape shape = CSX_SHAPE_BOX;
+  csx_boundary bc = CSX_BC_FIXED;
+  std::vector<double> w;           // base weights (2r+1)^ndim
+  int nnz = 0;
+  int tf = 1;                      // main fusion depth
+  int halo = 0;                    // r * tf
+  csx_engine engine_req = CSX_ENGINE_AUTO;
+  csx_engine engine = CSX_ENGINE_TC_S2R;
+  std::vector<csx::Pass> passes;   // index tf' - 1, for tf' = 1..tf
+  // device state (allocated at the first run)
+  int device = -1;
+  csx::Padded pad;
+  double* d_buf[2] = {nullptr, nullptr};
+  double* d_wbase = nullptr;       // base weights (direct engine, fix-up)
+  // sharded state
+  csx::Padded spad;                // per-rank slab grid
+  double* d_sbuf[2] = {nullptr, nullptr};
+  double* d_halo = nullptr;        // 4 halo staging slabs (send lo/hi, recv lo/hi)
+  int64_t s_lo = -1, s_hi = -1;
+  int s_rank = -1, s_nranks = 0;
+  int32_t* d_sband_tiles = nullptr;
+  int64_t sband_tiles_n = -1;
+  // FIXED band fix-up tiles of the single-GPU grid
+  int32_t* d_band_tiles = nullptr;
+  int64_t band_tiles_n = -1;
+  double* d_dense = nullptr;       // csx_run_host staging grid
+  // measurement hooks
+  bool prof = false;
+  std::vector<void*> prof_events;  // cudaEvent_t pairs around TC launches
+  size_t prof_used = 0;
+  int64_t n_tc_launches = 0, n_launches = 0;
+};
+
+namespace csx {
+// planner.cpp
+csx_status build_plan(csx_plan_s* p);
+csx_status build_pass(const csx_plan_s* p, int tf, Pass* out);
+void layout_padded(const csx_plan_s* p, const int64_t* E, Padded* pd);
+}  // namespace csx

@@ -1,0 +1,56 @@
+// kernels.cuh — device-side argument blocks and launcher declarations (product code).
+#pragma once
+#include <cuda_runtime.h>
+#include <cstdint>
+
+namespace csx {
+
+// A grid view: pointer at the interior origin plus strides of axes 0 and 1 (axis 2 stride 1).
+struct View {
+  double* p;
+  int64_t s0, s1;
+};
+struct CView {
+  const double* p;
+  int64_t s0, s1;
+};
+
+struct S2RArgs {
+  CView src;            // padded source (halo >= r*Tf readable around the interior)
+  View dst;             // destination (padded scratch or the user's dense d_out)
+  int64_t E0, E1, E2;   // interior extents (normalised, E0 slowest)
+  int tiles_x, tiles_y; // CTA tiles over (E2, E1) [2D: rows E1, cols E2]
+  int64_t ntiles;
+  const int2* lut;      // per region element {source offset, a | b << 16}
+  const double* frags;  // per-lane B fragments
+  const double* wc;     // composed weights (3D CUDA-core planes)
+};
+
+struct DirectArgs {
+  CView src;
+  View dst;
+  int64_t E[3];         // local interior extents
+  int64_t gorg[3];      // local origin in global coordinates (slab offset; 0 single-GPU)
+  int64_t GE[3];        // global extents (FIXED frame and band are global)
+  int real[3];          // 1 if the axis is a real (stencil) axis
+  int r, tf, fixed_bc;
+  int band;             // 0: write every point; >0: write only points within `band` of a face
+  int B[3];             // tile extents (outputs)
+  int tiles[3];
+  int64_t ntiles;
+  const int32_t* tile_list;  // band mode: linear tile ids; nullptr = all tiles
+  const double* w;      // base weights (2r+1)^ndim dense
+  int ndim;
+};
+
+// launchers (return cudaError_t of the launch)
+cudaError_t launch_pack(const double* in, View dst, const int64_t* E, cudaStream_t st);
+cudaError_t launch_ghost_fill(View buf, const int64_t* E, const int* real, const int* fill, int H,
+                              cudaStream_t st);
+cudaError_t launch_s2r(int ndim, int nk, int nf, const S2RArgs& a, int tc_mask, cudaStream_t st);
+cudaError_t launch_tile(int ndim, int nk, const S2RArgs& a, cudaStream_t st);
+cudaError_t launch_direct(const DirectArgs& a, cudaStream_t st);
+int s2r_smem_bytes(int ndim, int nk, int nf);
+int num_sms();
+
+}  // namespace csx

@@ -1,0 +1,351 @@
+// kernels_s2r.cu — the paper's design on sm_100a DMMA (engine TC_S2R).
+//
+// Per CTA tile (persistent CTAs, one LUT load per CTA):
+//   a4  implicit stencil2row: the input region is read once from HBM (coalesced along rows)
+//       and scattered through the lookup table into the stencil2row tiles A and B in shared
+//       memory; elements belonging to neither land in the dirty row — no branches
+//       (P.787-797, P.1711-1773, Fig 5).
+//   a5  dual tessellation: for each output row, acc(8x8) = Tile_A . W_A + Tile_B . W_B as one
+//       chain of 2*ceil(K/4) DMMA.8x8x4 (mma.sync m8n8k4 f64), vitrolite B accumulated onto A
+//       (P.900-959, P.1332-1336, P.1449-1461).  W_A/W_B fragments live in registers.
+//   a6  store: lane (g, t) holds outputs (x, g*(nk+1) + 2t + {0,1}) — the window centre
+//       (P.1326-1331): one warp writes 8*(nk+1) contiguous doubles.
+//   a8  1D: stencil2row rows of length nk, same dual tessellation, N fragments when nk+1 > 8.
+//   a9  3D: sum over z offsets of 2D ConvStencils with per-plane weights; single-tap planes
+//       (star arms) on CUDA cores in the same kernel (P.1788-1800).
+#include <cuda_runtime.h>
+
+#include "kernels.cuh"
+#include "s2r_geom.h"
+
+namespace csx {
+
+__device__ __forceinline__ void dmma(double& c0, double& c1, double a, double b) {
+  asm("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+      : "+d"(c0), "+d"(c1)
+      : "d"(a), "d"(b));
+}
+
+// Store the two accumulator values of one lane (columns col, col+1 of one output row).
+__device__ __forceinline__ void store_pair(double* row_ptr, int64_t col, int64_t ncols, bool v0,
+                                           bool v1, double c0, double c1) {
+  double* p = row_ptr + col;
+  if (v0 && v1 && col + 1 < ncols && ((reinterpret_cast<uintptr_t>(p) & 15) == 0)) {
+    *reinterpret_cast<double2*>(p) = make_double2(c0, c1);
+  } else {
+    if (v0 && col < ncols) p[0] = c0;
+    if (v1 && col + 1 < ncols) p[1] = c1;
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+// 2D
+template <int NK>
+__global__ void __launch_bounds__(128, 3) k_s2r2d(S2RArgs a) {
+  using G = S2R2D<NK>;
+  extern __shared__ __align__(16) double smem[];
+  double* sA = smem;
+  double* sB = smem + (G::STRIPS + 1) * G::PITCH;
+  int2* sL = reinterpret_cast<int2*>(smem + 2 * (G::STRIPS + 1) * G::PITCH);
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  // Zero the tiles once so that the K-padding and pad slots are finite (0 * weight 0 = 0).
+  for (int i = tid; i < 2 * (G::STRIPS + 1) * G::PITCH; i += G::NT) smem[i] = 0.0;
+  for (int i = tid; i < G::NE; i += G::NT) sL[i] = a.lut[i];
+  double wa[G::KS], wb[G::KS];
+#pragma unroll
+  for (int s = 0; s < G::KS; ++s) {
+    wa[s] = a.frags[s * 32 + lane];
+    wb[s] = a.frags[(G::KS + s) * 32 + lane];
+  }
+  const int g = lane >> 2, t = lane & 3;
+  const bool v0 = 2 * t < G::SW, v1 = 2 * t + 1 < G::SW;
+  for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x) {
+    const int ty = (int)(tile / a.tiles_x);
+    const int tx = (int)(tile - (int64_t)ty * a.tiles_x);
+    const double* base = a.src.p + (int64_t)(ty * G::BM - G::R) * a.src.s1 + (tx * G::BN - G::R);
+    __syncthreads();  // the previous tile's fragment reads are done
+#pragma unroll 7
+    for (int e = tid; e < G::NE; e += G::NT) {
+      const int2 l = sL[e];
+      const double v = __ldg(base + l.x);
+      sA[l.y & 0xffff] = v;
+      sB[((unsigned)l.y) >> 16] = v;
+    }
+    __syncthreads();
+    const int64_t col = (int64_t)tx * G::BN + g * G::SW + 2 * t;
+#pragma unroll 1
+    for (int xr = warp * (G::BM / 4); xr < (warp + 1) * (G::BM / 4); xr += 2) {
+      const double* pa = sA + g * G::PITCH + G::NKV * xr + t;
+      const double* pb = sB + g * G::PITCH + G::NKV * xr + t;
+      double c00 = 0.0, c01 = 0.0, c10 = 0.0, c11 = 0.0;
+#pragma unroll
+      for (int s = 0; s < G::KS; ++s) {
+        dmma(c00, c01, pa[4 * s], wa[s]);
+        dmma(c10, c11, pa[4 * s + G::NKV], wa[s]);
+      }
+#pragma unroll
+      for (int s = 0; s < G::KS; ++s) {
+        dmma(c00, c01, pb[4 * s], wb[s]);
+        dmma(c10, c11, pb[4 * s + G::NKV], wb[s]);
+      }
+      const int64_t row = (int64_t)ty * G::BM + xr;
+      if (row < a.E1) store_pair(a.dst.p + row * a.dst.s1, col, a.E2, v0, v1, c00, c01);
+      if (row + 1 < a.E1) store_pair(a.dst.p + (row + 1) * a.dst.s1, col, a.E2, v0, v1, c10, c11);
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+// 1D (P.1779-1786): stencil2row rows k hold X[k(nk+1) .. k(nk+1)+nk); one dual tessellation
+// covers 8 rows = 8 (nk+1) outputs; N fragments f cover output columns 8f .. 8f+7.
+template <int NK>
+__global__ void __launch_bounds__(128, 4) k_s2r1d(S2RArgs a) {
+  using G = S2R1D<NK>;
+  constexpr int NF = G::NF, KS = G::KS;
+  extern __shared__ __align__(16) double smem[];
+  double* sA = smem;
+  double* sB = smem + (G::STRIPS + 1) * G::PITCH;
+  int2* sL = reinterpret_cast<int2*>(smem + 2 * (G::STRIPS + 1) * G::PITCH);
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  for (int i = tid; i < 2 * (G::STRIPS + 1) * G::PITCH; i += G::NT) smem[i] = 0.0;
+  for (int i = tid; i < G::NE; i += G::NT) sL[i] = a.lut[i];
+  double wa[NF][KS], wb[NF][KS];
+#pragma unroll
+  for (int f = 0; f < NF; ++f)
+#pragma unroll
+    for (int s = 0; s < KS; ++s) {
+      wa[f][s] = a.frags[((0 * NF + f) * KS + s) * 32 + lane];
+      wb[f][s] = a.frags[((1 * NF + f) * KS + s) * 32 + lane];
+    }
+  const int g = lane >> 2, t = lane & 3;
+  for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x) {
+    const double* base = a.src.p + tile * G::BN - G::R;
+    __syncthreads();
+#pragma unroll 4
+    for (int e = tid; e < G::NE; e += G::NT) {
+      const int2 l = sL[e];
+      const double v = __ldg(base + l.x);
+      sA[l.y & 0xffff] = v;
+      sB[((unsigned)l.y) >> 16] = v;
+    }
+    __syncthreads();
+#pragma unroll 1
+    for (int d = warp; d < G::NDT; d += 4) {
+      const double* pa = sA + (8 * d + g) * G::PITCH + t;
+      const double* pb = sB + (8 * d + g) * G::PITCH + t;
+      double c[NF][2];
+#pragma unroll
+      for (int f = 0; f < NF; ++f) c[f][0] = c[f][1] = 0.0;
+#pragma unroll
+      for (int s = 0; s < KS; ++s) {
+        const double x = pa[4 * s];
+#pragma unroll
+        for (int f = 0; f < NF; ++f) dmma(c[f][0], c[f][1], x, wa[f][s]);
+      }
+#pragma unroll
+      for (int s = 0; s < KS; ++s) {
+        const double x = pb[4 * s];
+#pragma unroll
+        for (int f = 0; f < NF; ++f) dmma(c[f][0], c[f][1], x, wb[f][s]);
+      }
+      const int64_t o = tile * G::BN + (int64_t)(8 * d + g) * G::SW;
+#pragma unroll
+      for (int f = 0; f < NF; ++f) {
+        const int cc = 8 * f + 2 * t;
+        store_pair(a.dst.p, o + cc, a.E2, cc < G::SW, cc + 1 < G::SW, c[f][0], c[f][1]);
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+// 3D (Tf = 1): stream input planes along z; input plane zi contributes to output planes
+// zo = zi - R + j with the 2D weights of z offset dz = NK-1-j (P.1788-1800).  Accumulators of
+// the NK live output planes rotate in registers.  Planes whose weights are a single centre tap
+// (star arms) are applied with DFMA on CUDA cores from a raw copy of the region.
+template <int NK>
+__global__ void __launch_bounds__(128, 3) k_s2r3d(S2RArgs a, int tc_mask) {
+  using G = S2R3D<NK>;
+  constexpr int KS = G::KS, R = G::R;
+  extern __shared__ __align__(16) double smem[];
+  double* sA = smem;
+  double* sB = smem + (G::STRIPS + 1) * G::PITCH;
+  int2* sL = reinterpret_cast<int2*>(smem + 2 * (G::STRIPS + 1) * G::PITCH);
+  double* sX = reinterpret_cast<double*>(sL + G::NE);  // raw region (CUDA-core planes)
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  for (int i = tid; i < 2 * (G::STRIPS + 1) * G::PITCH; i += G::NT) smem[i] = 0.0;
+  for (int i = tid; i < G::NE; i += G::NT) sL[i] = a.lut[i];
+  double wa[NK][KS], wb[NK][KS], wz[NK];
+#pragma unroll
+  for (int p = 0; p < NK; ++p) {
+#pragma unroll
+    for (int s = 0; s < KS; ++s) {
+      wa[p][s] = a.frags[((p * 2 + 0) * KS + s) * 32 + lane];
+      wb[p][s] = a.frags[((p * 2 + 1) * KS + s) * 32 + lane];
+    }
+    wz[p] = a.wc[(p * NK + R) * NK + R];
+  }
+  const int g = lane >> 2, t = lane & 3;
+  const bool v0 = 2 * t < G::SW, v1 = 2 * t + 1 < G::SW;
+  const bool need_raw = tc_mask != (1 << NK) - 1;
+  const int64_t nz = (a.E0 + G::ZCHUNK - 1) / G::ZCHUNK;
+  const int64_t ncol = (int64_t)a.tiles_x * a.tiles_y;
+  for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
+    const int64_t zc = item / ncol;
+    const int64_t tile = item - zc * ncol;
+    const int ty = (int)(tile / a.tiles_x);
+    const int tx = (int)(tile - (int64_t)ty * a.tiles_x);
+    const int64_t z0 = zc * G::ZCHUNK;
+    const int64_t z1 = min(a.E0, z0 + G::ZCHUNK);
+    (void)nz;
+    const double* base2 = a.src.p + (int64_t)(ty * G::BM - R) * a.src.s1 + (tx * G::BN - R);
+    double acc[NK][2][2];
+#pragma unroll
+    for (int j = 0; j < NK; ++j) acc[j][0][0] = acc[j][0][1] = acc[j][1][0] = acc[j][1][1] = 0.0;
+    const int xr = warp * 2;
+    const int64_t col = (int64_t)tx * G::BN + g * G::SW + 2 * t;
+    for (int64_t zi = z0 - R; zi < z1 + R; ++zi) {
+      const double* base = base2 + zi * a.src.s0;
+      __syncthreads();
+#pragma unroll 4
+      for (int e = tid; e < G::NE; e += G::NT) {
+        const int2 l = sL[e];
+        const double v = __ldg(base + l.x);
+        sA[l.y & 0xffff] = v;
+        sB[((unsigned)l.y) >> 16] = v;
+        if (need_raw) sX[e] = v;
+      }
+      __syncthreads();
+      const double* pa = sA + g * G::PITCH + NK * xr + t;
+      const double* pb = sB + g * G::PITCH + NK * xr + t;
+#pragma unroll
+      for (int j = 0; j < NK; ++j) {
+        const int dz = NK - 1 - j;
+        if (tc_mask & (1 << dz)) {
+#pragma unroll
+          for (int s = 0; s < KS; ++s) {
+            dmma(acc[j][0][0], acc[j][0][1], pa[4 * s], wa[dz][s]);
+            dmma(acc[j][1][0], acc[j][1][1], pa[4 * s + NK], wa[dz][s]);
+          }
+#pragma unroll
+          for (int s = 0; s < KS; ++s) {
+            dmma(acc[j][0][0], acc[j][0][1], pb[4 * s], wb[dz][s]);
+            dmma(acc[j][1][0], acc[j][1][1], pb[4 * s + NK], wb[dz][s]);
+          }
+        } else if (wz[dz] != 0.0) {
+          // centre tap of output (xr + h, g*SW + 2t + e) is region (xr + h + R, g*SW + 2t + e + R)
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const double* px = sX + (xr + h + R) * G::RC + g * G::SW + 2 * t + R;
+            acc[j][h][0] = fma(wz[dz], px[0], acc[j][h][0]);
+            acc[j][h][1] = fma(wz[dz], px[1], acc[j][h][1]);
+          }
+        }
+      }
+      const int64_t zo = zi - R;
+      if (zo >= z0) {
+        double* plane = a.dst.p + zo * a.dst.s0;
+        const int64_t row = (int64_t)ty * G::BM + xr;
+        if (row < a.E1) store_pair(plane + row * a.dst.s1, col, a.E2, v0, v1, acc[0][0][0], acc[0][0][1]);
+        if (row + 1 < a.E1)
+          store_pair(plane + (row + 1) * a.dst.s1, col, a.E2, v0, v1, acc[0][1][0], acc[0][1][1]);
+      }
+#pragma unroll
+      for (int j = 0; j + 1 < NK; ++j) {
+        acc[j][0][0] = acc[j + 1][0][0]; acc[j][0][1] = acc[j + 1][0][1];
+        acc[j][1][0] = acc[j + 1][1][0]; acc[j][1][1] = acc[j + 1][1][1];
+      }
+      acc[NK - 1][0][0] = acc[NK - 1][0][1] = acc[NK - 1][1][0] = acc[NK - 1][1][1] = 0.0;
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+int num_sms() {
+  static int n = 0;
+  if (n == 0) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (n <= 0) n = 148;
+  }
+  return n;
+}
+
+template <class K>
+static cudaError_t launch_persistent(K kernel, int smem, int per_sm, int64_t items, cudaStream_t st,
+                                     const S2RArgs& a) {
+  cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e != cudaSuccess) return e;
+  int occ = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, 128, smem);
+  if (e != cudaSuccess) return e;
+  if (occ < 1) return cudaErrorInvalidConfiguration;
+  (void)per_sm;
+  int64_t grid = (int64_t)occ * num_sms();
+  if (grid > items) grid = items;
+  if (grid < 1) grid = 1;
+  kernel<<<(unsigned)grid, 128, smem, st>>>(a);
+  return cudaGetLastError();
+}
+
+int s2r_smem_bytes(int ndim, int nk, int nf) {
+  (void)nf;
+  if (ndim == 1) {
+    switch (nk) {
+      case 3: return S2R1D<3>::SMEM;
+      case 5: return S2R1D<5>::SMEM;
+      case 7: return S2R1D<7>::SMEM;
+      case 9: return S2R1D<9>::SMEM;
+      case 11: return S2R1D<11>::SMEM;
+      case 13: return S2R1D<13>::SMEM;
+      case 15: return S2R1D<15>::SMEM;
+    }
+  } else if (ndim == 2) {
+    switch (nk) {
+      case 3: return S2R2D<3>::SMEM;
+      case 5: return S2R2D<5>::SMEM;
+      case 7: return S2R2D<7>::SMEM;
+    }
+  } else if (nk == 3) {
+    return S2R3D<3>::SMEM;
+  }
+  return -1;
+}
+
+cudaError_t launch_s2r(int ndim, int nk, int nf, const S2RArgs& a, int tc_mask, cudaStream_t st) {
+  (void)nf;
+  const int smem = s2r_smem_bytes(ndim, nk, nf);
+  if (smem < 0) return cudaErrorInvalidValue;
+  if (ndim == 1) {
+    switch (nk) {
+      case 3: return launch_persistent(k_s2r1d<3>, smem, 4, a.ntiles, st, a);
+      case 5: return launch_persistent(k_s2r1d<5>, smem, 4, a.ntiles, st, a);
+      case 7: return launch_persistent(k_s2r1d<7>, smem, 4, a.ntiles, st, a);
+      case 9: return launch_persistent(k_s2r1d<9>, smem, 4, a.ntiles, st, a);
+      case 11: return launch_persistent(k_s2r1d<11>, smem, 4, a.ntiles, st, a);
+      case 13: return launch_persistent(k_s2r1d<13>, smem, 4, a.ntiles, st, a);
+      case 15: return launch_persistent(k_s2r1d<15>, smem, 4, a.ntiles, st, a);
+    }
+  } else if (ndim == 2) {
+    switch (nk) {
+      case 3: return launch_persistent(k_s2r2d<3>, smem, 3, a.ntiles, st, a);
+      case 5: return launch_persistent(k_s2r2d<5>, smem, 3, a.ntiles, st, a);
+      case 7: return launch_persistent(k_s2r2d<7>, smem, 3, a.ntiles, st, a);
+    }
+  } else if (nk == 3) {
+    auto kern = k_s2r3d<3>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    int occ = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 128, smem);
+    if (e != cudaSuccess) return e;
+    int64_t grid = (int64_t)(occ < 1 ? 1 : occ) * num_sms();
+    if (grid > a.ntiles) grid = a.ntiles;
+    kern<<<(unsigned)grid, 128, smem, st>>>(a, tc_mask);
+    return cudaGetLastError();
+  }
+  return cudaErrorInvalidValue;
+}
+
+}  // namespace csx
