@@ -166,21 +166,22 @@ csx_status csx_run_sharded(csx_plan_t p, csx_comm_t c, const double* d_in, doubl
   if (p->s_rank != c->rank || p->s_nranks != c->nranks) {
     cudaFree(p->d_sbuf[0]);
     cudaFree(p->d_sbuf[1]);
-    cudaFree(p->d_sband_tiles);
     p->d_sbuf[0] = p->d_sbuf[1] = nullptr;
-    p->d_sband_tiles = nullptr;
-    p->sband_tiles_n = 0;
+    if (p->sstrips) {
+      free_strips(static_cast<StripSet*>(p->sstrips), p->nsstrips);
+      delete[] static_cast<StripSet*>(p->sstrips);
+      p->sstrips = nullptr;
+    }
+    p->nsstrips = 0;
     s = ensure_grid(p, &p->spad, p->d_sbuf, El);
     if (s != CSX_OK) return s;
     if (p->bc == CSX_BC_FIXED) {
       int64_t gorg[3] = {0, 0, 0};
       gorg[a0] = lo;
-      std::vector<int32_t> bt = band_tiles(p->ndim, El, gorg, p->E, p->halo);
-      p->sband_tiles_n = (int64_t)bt.size();
-      cudaError_t e = cudaMalloc(&p->d_sband_tiles, (bt.size() + 1) * sizeof(int32_t));
-      if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc");
-      e = cudaMemcpy(p->d_sband_tiles, bt.data(), bt.size() * sizeof(int32_t), cudaMemcpyHostToDevice);
-      if (e != cudaSuccess) return cuda_fail(e, "upload band tiles");
+      StripSet* ss = new StripSet[2];
+      p->sstrips = ss;
+      s = build_strips(p->ndim, El, gorg, p->E, p->halo, ss, &p->nsstrips);
+      if (s != CSX_OK) return s;
     }
     p->s_rank = c->rank;
     p->s_nranks = c->nranks;
@@ -219,8 +220,8 @@ csx_status csx_run_sharded(csx_plan_t p, csx_comm_t c, const double* d_in, doubl
     pc.dst = last ? out : b[cur ^ 1];
     for (int a = 0; a < 3; ++a) { pc.E[a] = El[a]; pc.gorg[a] = 0; }
     pc.gorg[a0] = lo;
-    pc.band_tiles = p->d_sband_tiles;
-    pc.n_band_tiles = p->sband_tiles_n;
+    pc.strips = static_cast<const StripSet*>(p->sstrips);
+    pc.nstrips = p->nsstrips < 0 ? 0 : p->nsstrips;
     s = run_pass(p, p->passes[tfp - 1], pc, st);
     if (s != CSX_OK) return s;
     if (!last) {

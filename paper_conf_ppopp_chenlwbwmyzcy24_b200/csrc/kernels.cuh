@@ -39,6 +39,7 @@ struct DirectArgs {
   int tiles[3];
   int64_t ntiles;
   const int32_t* tile_list;  // band mode: linear tile ids; nullptr = all tiles
+  const int64_t* tile_org;   // band strips: explicit tile origins (3 per tile), or nullptr
   const double* w;      // base weights (2r+1)^ndim dense
   int ndim;
 };
@@ -50,6 +51,10 @@ cudaError_t launch_ghost_fill(View buf, const int64_t* E, const int* real, const
 cudaError_t launch_s2r(int ndim, int nk, int nf, const S2RArgs& a, int tc_mask, cudaStream_t st);
 cudaError_t launch_tile(int ndim, int nk, const S2RArgs& a, cudaStream_t st);
 cudaError_t launch_direct(const DirectArgs& a, cudaStream_t st);
+// FIXED frame (points within r of a GLOBAL face) copied src -> dst: the whole fix-up of a
+// Tf = 1 pass, whose composed window is the plain stencil (no band beyond the frame).
+cudaError_t launch_frame_copy(CView src, View dst, const int64_t* E, const int64_t* gorg,
+                              const int64_t* GE, const int* real, int r, cudaStream_t st);
 int s2r_smem_bytes(int ndim, int nk, int nf);
 int num_sms();
 

@@ -48,13 +48,20 @@ __global__ void __launch_bounds__(256) k_direct(DirectArgs a) {
   __syncthreads();
   const int nt = ntaps;
   for (int64_t it = blockIdx.x; it < a.ntiles; it += gridDim.x) {
-    const int64_t tid_lin = a.tile_list ? (int64_t)a.tile_list[it] : it;
-    const int64_t t2 = tid_lin % a.tiles[2];
-    const int64_t t1 = (tid_lin / a.tiles[2]) % a.tiles[1];
-    const int64_t t0 = tid_lin / ((int64_t)a.tiles[2] * a.tiles[1]);
-    const int64_t o0 = t0 * a.B[0] - (a.real[0] ? h : 0);
-    const int64_t o1 = t1 * a.B[1] - (a.real[1] ? h : 0);
-    const int64_t o2 = t2 * a.B[2] - h;
+    int64_t b0, b1, b2;  // tile origin (local coordinates of its first output)
+    if (a.tile_org) {
+      b0 = a.tile_org[3 * it];
+      b1 = a.tile_org[3 * it + 1];
+      b2 = a.tile_org[3 * it + 2];
+    } else {
+      const int64_t tid_lin = a.tile_list ? (int64_t)a.tile_list[it] : it;
+      b2 = (tid_lin % a.tiles[2]) * a.B[2];
+      b1 = ((tid_lin / a.tiles[2]) % a.tiles[1]) * a.B[1];
+      b0 = (tid_lin / ((int64_t)a.tiles[2] * a.tiles[1])) * a.B[0];
+    }
+    const int64_t o0 = b0 - (a.real[0] ? h : 0);
+    const int64_t o1 = b1 - (a.real[1] ? h : 0);
+    const int64_t o2 = b2 - h;
     // load the region (halo h on real axes) from the padded source
     for (int row = warp; row < RB0 * RB1; row += nw) {
       const int z = row / RB1, y = row - z * RB1;
@@ -99,7 +106,7 @@ __global__ void __launch_bounds__(256) k_direct(DirectArgs a) {
     const int h0 = a.real[0] ? h : 0, h1 = a.real[1] ? h : 0;
     for (int row = warp; row < a.B[0] * a.B[1]; row += nw) {
       const int z = row / a.B[1], y = row - z * a.B[1];
-      const int64_t lz = t0 * a.B[0] + z, ly = t1 * a.B[1] + y;  // local coordinates
+      const int64_t lz = b0 + z, ly = b1 + y;  // local coordinates
       if (lz >= a.E[0] || ly >= a.E[1]) continue;
       const int64_t gz = a.gorg[0] + lz, gy = a.gorg[1] + ly;
       const bool rowband = (a.real[0] && (gz < a.band || gz >= a.GE[0] - a.band)) ||
@@ -107,7 +114,7 @@ __global__ void __launch_bounds__(256) k_direct(DirectArgs a) {
       const double* src = in + ((z + h0) * RB1 + (y + h1)) * RB2 + h;
       double* dst = a.dst.p + lz * a.dst.s0 + ly * a.dst.s1;
       for (int x = lane; x < a.B[2]; x += 32) {
-        const int64_t lx = t2 * a.B[2] + x;
+        const int64_t lx = b2 + x;
         if (lx >= a.E[2]) continue;
         const int64_t gx = a.gorg[2] + lx;
         if (a.band > 0 && !(rowband || gx < a.band || gx >= a.GE[2] - a.band)) continue;
@@ -156,6 +163,37 @@ cudaError_t launch_direct(const DirectArgs& a, cudaStream_t st) {
 }
 
 // ------------------------------------------------------------------------------------------
+__global__ void k_frame_copy(CView src, View dst, int64_t E0, int64_t E1, int64_t E2, int64_t g0,
+                             int64_t g1, int64_t g2, int64_t G0, int64_t G1, int64_t G2, int real0,
+                             int real1, int r) {
+  const int64_t nrows = E0 * E1;
+  for (int64_t row = blockIdx.x; row < nrows; row += gridDim.x) {
+    const int64_t z = row / E1, y = row - z * E1;
+    const int64_t gz = g0 + z, gy = g1 + y;
+    const bool whole = (real0 && (gz < r || gz >= G0 - r)) || (real1 && (gy < r || gy >= G1 - r));
+    const double* s = src.p + z * src.s0 + y * src.s1;
+    double* d = dst.p + z * dst.s0 + y * dst.s1;
+    if (whole) {
+      for (int64_t x = threadIdx.x; x < E2; x += blockDim.x) d[x] = s[x];
+    } else {
+      for (int64_t k = threadIdx.x; k < 2 * r; k += blockDim.x) {
+        const int64_t gx = k < r ? k : G2 - 2 * r + k;  // global frame column
+        const int64_t x = gx - g2;
+        if (x >= 0 && x < E2) d[x] = s[x];
+      }
+    }
+  }
+}
+
+cudaError_t launch_frame_copy(CView src, View dst, const int64_t* E, const int64_t* gorg,
+                              const int64_t* GE, const int* real, int r, cudaStream_t st) {
+  const int64_t nrows = E[0] * E[1];
+  const int64_t grid = nrows < 8 * num_sms() ? nrows : 8 * num_sms();
+  k_frame_copy<<<(unsigned)grid, 128, 0, st>>>(src, dst, E[0], E[1], E[2], gorg[0], gorg[1], gorg[2],
+                                               GE[0], GE[1], GE[2], real[0], real[1], r);
+  return cudaGetLastError();
+}
+
 __global__ void k_pack(const double* __restrict__ in, View dst, int64_t E1, int64_t E2,
                        int64_t nrows) {
   for (int64_t row = blockIdx.x; row < nrows; row += gridDim.x) {

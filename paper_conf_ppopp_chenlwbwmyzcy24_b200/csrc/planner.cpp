@@ -109,16 +109,16 @@ int choose_pitch(int min_pitch) {
 void layout_padded(const csx_plan_s* p, const int64_t* E, Padded* pd) {
   const int H = p->halo;
   const int real0 = p->ndim == 3, real1 = p->ndim >= 2;
-  // worst-case tile over-read beyond the interior (tiles are rounded up to the CTA tile)
-  const int64_t tile_r = 64, tile_c = 128;
+  // slack beyond the interior for CTA tiles that overhang the last row / column (every
+  // kernel's tile is <= 128 rows and <= 128 + 32 columns including its halo)
   for (int a = 0; a < 3; ++a) pd->E[a] = E[a];
   pd->O[0] = real0 ? H : 0;
   pd->O[1] = real1 ? H : 0;
   pd->O[2] = 16 * ((H + 15) / 16);  // >= H, interior rows 128-byte aligned
   if (pd->O[2] < 16) pd->O[2] = 16;
   pd->A[0] = real0 ? (E[0] + 2 * H + 2) : 1;
-  pd->A[1] = real1 ? (pd->O[1] + ((E[1] + tile_r - 1) / tile_r) * tile_r + H + 2) : 1;
-  const int64_t need2 = pd->O[2] + ((E[2] + tile_c - 1) / tile_c) * tile_c + H + 32;
+  pd->A[1] = real1 ? (pd->O[1] + E[1] + 128 + H + 2) : 1;
+  const int64_t need2 = pd->O[2] + E[2] + 160 + H + 32;
   pd->A[2] = 32 * ((need2 + 31) / 32);
   pd->s1 = pd->A[2];
   pd->s0 = pd->A[1] * pd->A[2];

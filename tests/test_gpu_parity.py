@@ -48,7 +48,7 @@ TSTEPS = {1: 17, 2: 7, 3: 3}
 
 @pytest.mark.parametrize("name", list(synth.SHAPES))
 @pytest.mark.parametrize("bc", ["fixed", "periodic"])
-@pytest.mark.parametrize("engine", ["tc_s2r", "direct"])
+@pytest.mark.parametrize("engine", ["tc_s2r", "tc_tile", "direct"])
 def test_parity_small(csx, name, bc, engine):
     s = synth.SHAPES[name]
     ext = SMALL[s.ndim]
@@ -68,11 +68,12 @@ def test_parity_small(csx, name, bc, engine):
 
 @pytest.mark.parametrize("tf", [1, 2, 3])
 @pytest.mark.parametrize("bc", ["fixed", "periodic"])
-def test_parity_fusion_depths_2d(csx, tf, bc):
+@pytest.mark.parametrize("engine", ["tc_s2r", "tc_tile"])
+def test_parity_fusion_depths_2d(csx, tf, bc, engine):
     u0 = synth.grid((67, 130), seed=5)
     w = synth.random_weights("box2d9p")
     for T in (1, 2, 3, 4, 5, 10):
-        got, info = run_gpu(csx, u0, w, "box", bc, T, engine="tc_s2r", fuse_steps=tf)
+        got, info = run_gpu(csx, u0, w, "box", bc, T, engine=engine, fuse_steps=tf)
         assert info["fuse_steps"] == tf
         assert rel(got, oracle.run(u0, w, bc, T)) <= TOL, (tf, T)
 
@@ -91,8 +92,9 @@ def test_signed_weights_general_radius(csx):
         w = synth.random_signed_weights(ndim, r, seed=9)
         u0 = synth.grid(ext, seed=10)
         for bc in ("fixed", "periodic"):
-            got, _ = run_gpu(csx, u0, w, "box", bc, 4, engine="tc_s2r")
-            assert rel(got, oracle.run(u0, w, bc, 4)) <= TOL, (ndim, r, bc)
+            for engine in ("tc_s2r", "auto"):
+                got, _ = run_gpu(csx, u0, w, "box", bc, 4, engine=engine)
+                assert rel(got, oracle.run(u0, w, bc, 4)) <= TOL, (ndim, r, bc, engine)
 
 
 def test_edge_cases(csx):
@@ -149,6 +151,7 @@ def test_full_size_sampled_box2d9p(csx):
     w = synth.random_weights("box2d9p")
     u0 = synth.grid(ext)
     got, info = run_gpu(csx, u0, w, "box", "fixed", T)
+    assert info["engine_name"] == "tc_tile"  # bench.py's default engine for this config
     rng = np.random.default_rng(0)
     pts = [(int(rng.integers(0, ext[0])), int(rng.integers(0, ext[1]))) for _ in range(24)]
     pts += [(0, 0), (1, 1), (2, 5), (3, 3), (10239, 10239), (10237, 4000), (5000, 10238), (64, 63)]
