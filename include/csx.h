@@ -105,6 +105,13 @@ csx_status csx_nccl_unique_id(void* out128);
 /* Rows [lo, hi) of the slowest axis owned by `rank`: lo = floor(rank*N0/nranks). */
 csx_status csx_shard_rows(const csx_plan_t plan, int rank, int nranks, int64_t* lo, int64_t* hi);
 
+/* The halo-exchange schedule csx_run_sharded posts before every pass (host logic, no GPU).
+ * Writes up to 4 ops of 4 int64 each into ops: {kind (0 send, 1 recv), peer rank, first slab
+ * row (local interior index; negative = top ghost rows, >= local rows = bottom ghost rows),
+ * number of rows (= r*Tf)} in posting order (send down, recv up, send up, recv down), and
+ * their count into *nops.  PERIODIC closes the ring; FIXED end ranks skip the missing side. */
+csx_status csx_halo_schedule(const csx_plan_t plan, int rank, int nranks, int64_t* ops, int* nops);
+
 /* Slab-sharded run: the plan describes the GLOBAL grid; d_in_local / d_out_local hold this
  * rank's rows [lo, hi) (csx_shard_rows) x the other extents.  Halos of depth r*Tf are exchanged
  * with NCCL send/recv every pass (ring for PERIODIC).  Every rank must call with equal plan

@@ -80,7 +80,9 @@ _sig("csx_plan_lut", ctypes.c_int, [_vp, _i32p, _i32p, _i64p, ctypes.POINTER(cty
 _sig("csx_profile_enable", ctypes.c_int, [_vp, ctypes.c_int])
 _sig("csx_profile_read", ctypes.c_int, [_vp, ctypes.POINTER(ctypes.c_double), _i64p, _i64p, ctypes.c_int])
 
-EXPORTED = ["csx_profile_enable", "csx_profile_read", "csx_plan", "csx_plan_set_engine", "csx_run", "csx_run_host", "csx_comm_create",
+_sig("csx_halo_schedule", ctypes.c_int, [_vp, ctypes.c_int, ctypes.c_int, _i64p, ctypes.POINTER(ctypes.c_int)])
+
+EXPORTED = ["csx_halo_schedule", "csx_profile_enable", "csx_profile_read", "csx_plan", "csx_plan_set_engine", "csx_run", "csx_run_host", "csx_comm_create",
             "csx_comm_destroy", "csx_nccl_unique_id", "csx_shard_rows", "csx_run_sharded",
             "csx_plan_destroy", "csx_status_string", "csx_last_error", "csx_plan_info",
             "csx_compose_weights", "csx_weight_matrices", "csx_stencil2row_index",
@@ -245,6 +247,16 @@ def csx_shard_rows(plan, rank: int, nranks: int):
     return lo.value, hi.value
 
 
+def csx_halo_schedule(plan, rank: int, nranks: int):
+    """[(kind 'send'|'recv', peer, first_row, nrows), ...] in posting order."""
+    ops = np.zeros(16, dtype=np.int64)
+    n = ctypes.c_int()
+    _check(_lib.csx_halo_schedule(plan, rank, nranks, ops.ctypes.data_as(_i64p), ctypes.byref(n)),
+           "csx_halo_schedule")
+    return [("send" if ops[4 * k] == 0 else "recv", int(ops[4 * k + 1]), int(ops[4 * k + 2]),
+             int(ops[4 * k + 3])) for k in range(n.value)]
+
+
 def csx_run_sharded(plan, comm, d_in, d_out, timesteps: int, n_local: int, stream=None):
     _check(_lib.csx_run_sharded(plan, comm, _device_ptr(d_in, n_local, "d_in"),
                                 _device_ptr(d_out, n_local, "d_out"), int(timesteps),
@@ -295,6 +307,9 @@ class Plan:
 
     def run_sharded(self, comm, d_in, d_out, timesteps: int, n_local: int, stream=None):
         csx_run_sharded(self._h, comm, d_in, d_out, timesteps, n_local, stream)
+
+    def halo_schedule(self, rank: int, nranks: int):
+        return csx_halo_schedule(self._h, rank, nranks)
 
     def lut(self):
         return csx_plan_lut(self._h)

@@ -42,62 +42,6 @@ void direct_tile(int ndim, int* B) {
   else { B[0] = 8; B[1] = 8; B[2] = 32; }
 }
 
-static csx_status upload_strip(StripSet* ss, const std::vector<int64_t>& org) {
-  ss->n = (int64_t)org.size() / 3;
-  CSX_CUDA(cudaMalloc(&ss->d_org, std::max<size_t>(3, org.size()) * sizeof(int64_t)), "cudaMalloc(strips)");
-  if (!org.empty())
-    CSX_CUDA(cudaMemcpy(ss->d_org, org.data(), org.size() * sizeof(int64_t), cudaMemcpyHostToDevice),
-             "upload strips");
-  return CSX_OK;
-}
-
-// Strips of direct-kernel tiles that cover every point within `band` of a GLOBAL face of the
-// local grid (E = local extents, gorg = local origin in global coordinates, GE = global
-// extents).  2D: horizontal strips (band x 64) along the top / bottom rows, vertical strips
-// (32 x max(band, 32-2*band)) along the left / right columns.  1D: one 1024-tile at each end.
-// 3D runs Tf = 1 only, whose fix-up is the frame copy (no strips).
-csx_status build_strips(int ndim, const int64_t* E, const int64_t* gorg, const int64_t* GE, int band,
-                        StripSet* out, int* n) {
-  *n = 0;
-  if (ndim == 1) {
-    std::vector<int64_t> org;
-    const int64_t w = 1024;
-    if (gorg[2] == 0) { org.push_back(0); org.push_back(0); org.push_back(0); }
-    if (gorg[2] + E[2] == GE[2]) { org.push_back(0); org.push_back(0); org.push_back(std::max<int64_t>(0, E[2] - w)); }
-    out[0].B[0] = 1; out[0].B[1] = 1; out[0].B[2] = (int)w;
-    csx_status s = upload_strip(&out[0], org);
-    if (s != CSX_OK) return s;
-    *n = 1;
-  } else if (ndim == 2) {
-    std::vector<int64_t> h, v;
-    const int wh = 64, hv = 32, wv = std::max(band, 32 - 2 * band);
-    for (int64_t x = 0; x < E[2]; x += wh) {
-      if (gorg[1] == 0) { h.push_back(0); h.push_back(0); h.push_back(x); }
-      if (gorg[1] + E[1] == GE[1]) { h.push_back(0); h.push_back(std::max<int64_t>(0, E[1] - band)); h.push_back(x); }
-    }
-    for (int64_t y = 0; y < E[1]; y += hv) {
-      v.push_back(0); v.push_back(y); v.push_back(0);
-      v.push_back(0); v.push_back(y); v.push_back(std::max<int64_t>(0, E[2] - wv));
-    }
-    out[0].B[0] = 1; out[0].B[1] = band; out[0].B[2] = wh;
-    out[1].B[0] = 1; out[1].B[1] = hv; out[1].B[2] = wv;
-    csx_status s = upload_strip(&out[0], h);
-    if (s != CSX_OK) return s;
-    s = upload_strip(&out[1], v);
-    if (s != CSX_OK) return s;
-    *n = 2;
-  }
-  return CSX_OK;
-}
-
-void free_strips(StripSet* s, int n) {
-  for (int i = 0; i < n; ++i) {
-    cudaFree(s[i].d_org);
-    s[i].d_org = nullptr;
-    s[i].n = 0;
-  }
-}
-
 static csx_status upload_pass(Pass& ps) {
   if (ps.uploaded) return CSX_OK;
   if (ps.s2r_ok) {
@@ -187,6 +131,17 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
     a.wc = ps.d_wc;
     if (eng == CSX_ENGINE_TC_TILE) {
       a.frags = ps.d_tile_frags;
+      if (p->ndim == 3)
+        for (int dz = 0; dz < ps.nk; ++dz) a.tc_mask |= ps.plane_is_tc[dz] << dz;
+      if (p->bc == CSX_BC_FIXED && p->ndim == 2) {  // band fix-up fused into the edge CTAs
+        a.fix_band = p->radius * ps.tf;
+        a.r = p->radius;
+        a.wbase = p->d_wbase;
+        a.gorg1 = c.gorg[1];
+        a.gorg2 = c.gorg[2];
+        a.GE1 = p->E[1];
+        a.GE2 = p->E[2];
+      }
       e = launch_tile(p->ndim, ps.nk, a, st);
     } else {
       a.frags = ps.d_frags;
@@ -214,11 +169,7 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
   }
   const bool direct_all = eng == CSX_ENGINE_DIRECT;
   const int real[3] = {p->ndim == 3, p->ndim >= 2, 1};
-  if (!direct_all && p->bc == CSX_BC_FIXED && ps.tf == 1) {
-    e = launch_frame_copy(c.src, c.dst, c.E, c.gorg, p->E, real, p->radius, st);
-    if (e != cudaSuccess) return cuda_fail(e, "frame copy launch");
-    p->n_launches += 1;
-  } else if (direct_all || p->bc == CSX_BC_FIXED) {
+  if (direct_all) {
     DirectArgs d;
     d.src = c.src;
     d.dst = c.dst;
@@ -235,26 +186,28 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
     d.ndim = p->ndim;
     d.tile_list = nullptr;
     d.tile_org = nullptr;
-    if (direct_all) {
-      d.band = 0;
-      direct_tile(p->ndim, d.B);
-      for (int a2 = 0; a2 < 3; ++a2) d.tiles[a2] = (int)((c.E[a2] + d.B[a2] - 1) / d.B[a2]);
-      d.ntiles = (int64_t)d.tiles[0] * d.tiles[1] * d.tiles[2];
+    d.band = 0;
+    direct_tile(p->ndim, d.B);
+    for (int a2 = 0; a2 < 3; ++a2) d.tiles[a2] = (int)((c.E[a2] + d.B[a2] - 1) / d.B[a2]);
+    d.ntiles = (int64_t)d.tiles[0] * d.tiles[1] * d.tiles[2];
+    if (p->ndim == 2 && direct2d_exists(p->radius, ps.tf))
+      e = launch_direct2d(d, p->w.data(), st);
+    else
       e = launch_direct(d, st);
-      if (e != cudaSuccess) return cuda_fail(e, "direct launch");
+    if (e != cudaSuccess) return cuda_fail(e, "direct launch");
+    p->n_launches += 1;
+  } else if (p->bc == CSX_BC_FIXED) {
+    if (ps.tf == 1 || p->ndim == 3) {
+      // the composed window is the plain stencil: only the held frame needs restoring
+      e = launch_frame_copy(c.src, c.dst, c.E, c.gorg, p->E, real, p->radius, st);
+      if (e != cudaSuccess) return cuda_fail(e, "frame copy launch");
       p->n_launches += 1;
     } else {
-      d.band = p->radius * ps.tf;
-      for (int k = 0; k < c.nstrips; ++k) {
-        const StripSet& ss = c.strips[k];
-        if (ss.n == 0) continue;
-        for (int a2 = 0; a2 < 3; ++a2) { d.B[a2] = ss.B[a2]; d.tiles[a2] = 1; }
-        d.tile_org = ss.d_org;
-        d.ntiles = ss.n;
-        e = launch_direct(d, st);
-        if (e != cudaSuccess) return cuda_fail(e, "band fix-up launch");
-        p->n_launches += 1;
-      }
+      int launched = 0;
+      e = launch_band(p->ndim, p->radius, ps.tf, c.src, c.dst, c.E, c.gorg, p->E, p->w.data(), st,
+                      &launched);
+      if (e != cudaSuccess) return cuda_fail(e, "band fix-up launch");
+      p->n_launches += launched;
     }
   }
   return CSX_OK;
@@ -372,13 +325,6 @@ csx_status csx_run(csx_plan_t p, const double* d_in, double* d_out, int64_t T, v
   }
   s = ensure_grid(p, &p->pad, p->d_buf, p->E);
   if (s != CSX_OK) return s;
-  if (p->bc == CSX_BC_FIXED && p->nstrips < 0) {
-    const int64_t zero[3] = {0, 0, 0};
-    StripSet* ss = new StripSet[2];
-    p->strips = ss;
-    s = build_strips(p->ndim, p->E, zero, p->E, p->halo, ss, &p->nstrips);
-    if (s != CSX_OK) return s;
-  }
   return run_local(p, d_in, d_out, T, st);
 }
 
@@ -447,8 +393,7 @@ csx_status csx_plan_destroy(csx_plan_t p) {
     cudaFree(p->d_dense);
     cudaFree(p->d_sbuf[0]);
     cudaFree(p->d_sbuf[1]);
-    if (p->strips) { free_strips(static_cast<StripSet*>(p->strips), p->nstrips); delete[] static_cast<StripSet*>(p->strips); }
-    if (p->sstrips) { free_strips(static_cast<StripSet*>(p->sstrips), p->nsstrips); delete[] static_cast<StripSet*>(p->sstrips); }
+
     cudaSetDevice(cur);
   }
   delete p;
@@ -546,8 +491,6 @@ csx_status run_local(csx_plan_s* p, const double* d_in, double* d_out, int64_t T
     c.src = CView{b[cur].p, b[cur].s0, b[cur].s1};
     c.dst = last ? out : b[cur ^ 1];
     for (int a = 0; a < 3; ++a) { c.E[a] = p->E[a]; c.gorg[a] = 0; }
-    c.strips = static_cast<const StripSet*>(p->strips);
-    c.nstrips = p->nstrips < 0 ? 0 : p->nstrips;
     csx_status s = run_pass(p, p->passes[tfp - 1], c, st);
     if (s != CSX_OK) return s;
     if (!last && p->bc == CSX_BC_PERIODIC) {

@@ -47,43 +47,45 @@ static void slab_rows(const Padded& pd, double* base, int a0, int64_t k, int h, 
   }
 }
 
-// Halo exchange along the slab axis.  Every rank posts, in this order: send its last h rows
-// down, receive its top ghost from up, send its first h rows up, receive its bottom ghost from
-// down.  With that fixed order the k-th message between any pair is matched correctly even when
-// up == down (two ranks, or one rank talking to itself on a PERIODIC ring).
-static csx_status exchange(csx_plan_s* p, csx_comm_s* c, double* base, int a0, int64_t El,
-                           cudaStream_t st) {
+// Halo-exchange schedule (csx_halo_schedule).  Every rank posts, in this order: send its last
+// h rows down, receive its top ghost from up, send its first h rows up, receive its bottom ghost
+// from down.  With that fixed order the k-th message between any pair is matched correctly even
+// when up == down (two ranks, or one rank talking to itself on a PERIODIC ring).
+static int halo_schedule(const csx_plan_s* p, int rank, int nranks, int64_t El, int64_t* ops) {
   const int h = p->halo;
   const bool periodic = p->bc == CSX_BC_PERIODIC;
-  int up = c->rank - 1, down = c->rank + 1;
+  int up = rank - 1, down = rank + 1;
   if (periodic) {
-    up = (up + c->nranks) % c->nranks;
-    down = down % c->nranks;
+    up = (up + nranks) % nranks;
+    down = down % nranks;
   } else {
     if (up < 0) up = -1;
-    if (down >= c->nranks) down = -1;
+    if (down >= nranks) down = -1;
   }
-  double *send_top, *send_bot, *recv_top, *recv_bot;
-  size_t n;
-  slab_rows(p->spad, base, a0, 0, h, &send_top, &n);
-  slab_rows(p->spad, base, a0, El - h, h, &send_bot, &n);
-  slab_rows(p->spad, base, a0, -h, h, &recv_top, &n);
-  slab_rows(p->spad, base, a0, El, h, &recv_bot, &n);
+  int n = 0;
+  auto op = [&](int kind, int peer, int64_t row) {
+    ops[4 * n] = kind; ops[4 * n + 1] = peer; ops[4 * n + 2] = row; ops[4 * n + 3] = h;
+    ++n;
+  };
+  if (down >= 0) op(0, down, El - h);
+  if (up >= 0) { op(1, up, -h); op(0, up, 0); }
+  if (down >= 0) op(1, down, El);
+  return n;
+}
+
+static csx_status exchange(csx_plan_s* p, csx_comm_s* c, double* base, int a0, int64_t El,
+                           cudaStream_t st) {
+  int64_t ops[16];
+  const int nops = halo_schedule(p, c->rank, c->nranks, El, ops);
   ncclResult_t r = ncclGroupStart();
   if (r != ncclSuccess) return nccl_fail(r, "ncclGroupStart");
-  if (down >= 0) {
-    r = ncclSend(send_bot, n, ncclDouble, down, c->comm, st);
-    if (r != ncclSuccess) return nccl_fail(r, "ncclSend");
-  }
-  if (up >= 0) {
-    r = ncclRecv(recv_top, n, ncclDouble, up, c->comm, st);
-    if (r != ncclSuccess) return nccl_fail(r, "ncclRecv");
-    r = ncclSend(send_top, n, ncclDouble, up, c->comm, st);
-    if (r != ncclSuccess) return nccl_fail(r, "ncclSend");
-  }
-  if (down >= 0) {
-    r = ncclRecv(recv_bot, n, ncclDouble, down, c->comm, st);
-    if (r != ncclSuccess) return nccl_fail(r, "ncclRecv");
+  for (int k = 0; k < nops; ++k) {
+    double* ptr;
+    size_t n;
+    slab_rows(p->spad, base, a0, ops[4 * k + 2], (int)ops[4 * k + 3], &ptr, &n);
+    if (ops[4 * k] == 0) r = ncclSend(ptr, n, ncclDouble, (int)ops[4 * k + 1], c->comm, st);
+    else r = ncclRecv(ptr, n, ncclDouble, (int)ops[4 * k + 1], c->comm, st);
+    if (r != ncclSuccess) return nccl_fail(r, ops[4 * k] == 0 ? "ncclSend" : "ncclRecv");
   }
   r = ncclGroupEnd();
   if (r != ncclSuccess) return nccl_fail(r, "ncclGroupEnd");
@@ -140,6 +142,16 @@ csx_status csx_shard_rows(const csx_plan_t p, int rank, int nranks, int64_t* lo,
   return CSX_OK;
 }
 
+csx_status csx_halo_schedule(const csx_plan_t p, int rank, int nranks, int64_t* ops, int* nops) {
+  if (!p || !ops || !nops || nranks < 1 || rank < 0 || rank >= nranks)
+    return fail(CSX_ERR_INVALID_ARGUMENT, "bad arguments");
+  int64_t lo, hi;
+  csx_status s = csx_shard_rows(p, rank, nranks, &lo, &hi);
+  if (s != CSX_OK) return s;
+  *nops = halo_schedule(p, rank, nranks, hi - lo, ops);
+  return CSX_OK;
+}
+
 csx_status csx_run_sharded(csx_plan_t p, csx_comm_t c, const double* d_in, double* d_out,
                            int64_t T, void* stream) {
   if (!p || !c || !d_in || !d_out) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL argument");
@@ -167,22 +179,8 @@ csx_status csx_run_sharded(csx_plan_t p, csx_comm_t c, const double* d_in, doubl
     cudaFree(p->d_sbuf[0]);
     cudaFree(p->d_sbuf[1]);
     p->d_sbuf[0] = p->d_sbuf[1] = nullptr;
-    if (p->sstrips) {
-      free_strips(static_cast<StripSet*>(p->sstrips), p->nsstrips);
-      delete[] static_cast<StripSet*>(p->sstrips);
-      p->sstrips = nullptr;
-    }
-    p->nsstrips = 0;
     s = ensure_grid(p, &p->spad, p->d_sbuf, El);
     if (s != CSX_OK) return s;
-    if (p->bc == CSX_BC_FIXED) {
-      int64_t gorg[3] = {0, 0, 0};
-      gorg[a0] = lo;
-      StripSet* ss = new StripSet[2];
-      p->sstrips = ss;
-      s = build_strips(p->ndim, El, gorg, p->E, p->halo, ss, &p->nsstrips);
-      if (s != CSX_OK) return s;
-    }
     p->s_rank = c->rank;
     p->s_nranks = c->nranks;
     p->s_lo = lo;
@@ -220,8 +218,6 @@ csx_status csx_run_sharded(csx_plan_t p, csx_comm_t c, const double* d_in, doubl
     pc.dst = last ? out : b[cur ^ 1];
     for (int a = 0; a < 3; ++a) { pc.E[a] = El[a]; pc.gorg[a] = 0; }
     pc.gorg[a0] = lo;
-    pc.strips = static_cast<const StripSet*>(p->sstrips);
-    pc.nstrips = p->nsstrips < 0 ? 0 : p->nsstrips;
     s = run_pass(p, p->passes[tfp - 1], pc, st);
     if (s != CSX_OK) return s;
     if (!last) {

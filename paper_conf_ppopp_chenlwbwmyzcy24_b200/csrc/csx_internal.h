@@ -108,11 +108,6 @@ struct csx_plan_s {
   double* d_halo = nullptr;        // 4 halo staging slabs (send lo/hi, recv lo/hi)
   int64_t s_lo = -1, s_hi = -1;
   int s_rank = -1, s_nranks = 0;
-  // FIXED band fix-up strips (csx_run.h StripSet) of the single-GPU grid and of the slab
-  void* strips = nullptr;          // StripSet[2]
-  int nstrips = -1;
-  void* sstrips = nullptr;
-  int nsstrips = -1;
   double* d_dense = nullptr;       // csx_run_host staging grid
   // measurement hooks
   bool prof = false;

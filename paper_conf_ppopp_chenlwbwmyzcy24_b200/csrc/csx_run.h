@@ -9,21 +9,12 @@
 
 namespace csx {
 
-// FIXED band fix-up work: direct-kernel tiles of shape B at explicit origins (device array).
-struct StripSet {
-  int B[3] = {1, 1, 1};
-  int64_t* d_org = nullptr;  // 3 int64 per tile
-  int64_t n = 0;
-};
-
 // Everything one fused pass needs to know about the grid it runs on.
 struct PassCtx {
   CView src;                      // padded source at its interior origin
   View dst;                       // destination at its interior origin
   int64_t E[3];                   // local interior extents (normalised)
   int64_t gorg[3];                // local origin in global coordinates (slab offset)
-  const StripSet* strips;         // FIXED: strips covering the global face bands
-  int nstrips;
 };
 
 csx_status cuda_fail(cudaError_t e, const char* where);
@@ -32,10 +23,6 @@ csx_status ensure_grid(csx_plan_s* p, Padded* pd, double** bufs, const int64_t* 
 csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st);
 csx_status run_local(csx_plan_s* p, const double* d_in, double* d_out, int64_t T, cudaStream_t st);
 void direct_tile(int ndim, int* B);
-// Build (and upload) the band strips of a local grid; band = r * Tf of the main pass.
-csx_status build_strips(int ndim, const int64_t* E, const int64_t* gorg, const int64_t* GE, int band,
-                        StripSet* out, int* n);
-void free_strips(StripSet* s, int n);
 bool tile_kernel_exists(int ndim, int nk);
 
 }  // namespace csx

@@ -24,6 +24,14 @@ struct S2RArgs {
   const int2* lut;      // per region element {source offset, a | b << 16}
   const double* frags;  // per-lane B fragments
   const double* wc;     // composed weights (3D CUDA-core planes)
+  // TC_TILE fused FIXED band fix-up (0 = none): edge CTAs recompute the points within
+  // fix_band = r*Tf of a GLOBAL face by Tf plain steps on CUDA cores from the staged tile.
+  int tc_mask = 0;                // 3D: bit dz set = z offset dz runs on tensor cores
+  int fix_band = 0;
+  int r = 0;
+  const double* wbase = nullptr;  // base weights (2r+1)^2
+  int64_t gorg1 = 0, gorg2 = 0;   // local origin in global coordinates
+  int64_t GE1 = 0, GE2 = 0;       // global extents
 };
 
 struct DirectArgs {
@@ -51,6 +59,13 @@ cudaError_t launch_ghost_fill(View buf, const int64_t* E, const int* real, const
 cudaError_t launch_s2r(int ndim, int nk, int nf, const S2RArgs& a, int tc_mask, cudaStream_t st);
 cudaError_t launch_tile(int ndim, int nk, const S2RArgs& a, cudaStream_t st);
 cudaError_t launch_direct(const DirectArgs& a, cudaStream_t st);
+// 2D comparator kernel (kernels_direct2d.cu): compile-time (r, Tf), weights by value.
+bool direct2d_exists(int r, int tf);
+cudaError_t launch_direct2d(const DirectArgs& a, const double* w_host, cudaStream_t st);
+// FIXED band fix-up after a fused pass of Tf > 1 steps (kernels_band.cu), 1D and 2D.
+cudaError_t launch_band(int ndim, int r, int tf, CView src, View dst, const int64_t* E,
+                        const int64_t* gorg, const int64_t* GE, const double* w_host,
+                        cudaStream_t st, int* launched);
 // FIXED frame (points within r of a GLOBAL face) copied src -> dst: the whole fix-up of a
 // Tf = 1 pass, whose composed window is the plain stencil (no band beyond the frame).
 cudaError_t launch_frame_copy(CView src, View dst, const int64_t* E, const int64_t* gorg,

@@ -39,18 +39,77 @@ __device__ __forceinline__ void store_pair(double* row_ptr, int64_t col, int64_t
 }
 
 // ------------------------------------------------------------------------------------------
-// 2D
+// 2D.  Persistent CTAs: warp NCW is a producer that streams each tile's raw input region into a
+// 2-stage smem ring with cp.async.bulk (mbarrier full/empty); the 8 consumer warps run the
+// paper's pipeline per tile: LUT scatter (smem raw -> stencil2row A/B, dirty row absorbs the
+// unused elements), then dual tessellation on DMMA, then the centre store.
+__device__ __forceinline__ uint32_t s2r_smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void s2r_mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(s2r_smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void s2r_mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n.reg .pred P1;\nWAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+      "@!P1 bra WAIT_%=;\n}\n" ::"r"(s2r_smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void s2r_mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(s2r_smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void s2r_issue_rows(const double* src, int64_t pitch, double* dst, int rows,
+                                               int tp, uint64_t* bar, int lane) {
+  if (lane == 0)
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(s2r_smem_u32(bar)),
+                 "r"((uint32_t)(rows * tp * 8))
+                 : "memory");
+  __syncwarp();
+  for (int r = lane; r < rows; r += 32)
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n" ::
+            "r"(s2r_smem_u32(dst + r * tp)),
+        "l"(src + (int64_t)r * pitch), "r"((uint32_t)(tp * 8)), "r"(s2r_smem_u32(bar))
+        : "memory");
+}
+
 template <int NK>
-__global__ void __launch_bounds__(128, 3) k_s2r2d(S2RArgs a) {
+__global__ void __launch_bounds__(S2R2D<NK>::NT, 2) k_s2r2d(S2RArgs a) {
   using G = S2R2D<NK>;
-  extern __shared__ __align__(16) double smem[];
-  double* sA = smem;
-  double* sB = smem + (G::STRIPS + 1) * G::PITCH;
-  int2* sL = reinterpret_cast<int2*>(smem + 2 * (G::STRIPS + 1) * G::PITCH);
+  extern __shared__ __align__(128) double smem[];
+  __shared__ __align__(8) uint64_t full[G::RAW_STAGES], empty[G::RAW_STAGES];
+  double* raw = smem;                                           // RAW_STAGES x RAW
+  double* sA = raw + G::RAW_STAGES * G::RAW;
+  double* sB = sA + (G::STRIPS + 1) * G::PITCH;
+  uint32_t* sL = reinterpret_cast<uint32_t*>(sB + (G::STRIPS + 1) * G::PITCH);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  // Zero the tiles once so that the K-padding and pad slots are finite (0 * weight 0 = 0).
-  for (int i = tid; i < 2 * (G::STRIPS + 1) * G::PITCH; i += G::NT) smem[i] = 0.0;
-  for (int i = tid; i < G::NE; i += G::NT) sL[i] = a.lut[i];
+  constexpr int NC = G::NCW * 32;
+  // Zero the tiles once so that the K-padding and pad slots are finite (0 * weight 0 = 0);
+  // the LUT packs the A and B offsets of each region element (P.1711-1721).
+  for (int i = tid; i < 2 * (G::STRIPS + 1) * G::PITCH; i += G::NT) sA[i] = 0.0;
+  for (int i = tid; i < G::NE; i += G::NT) sL[i] = (uint32_t)a.lut[i].y;
+  if (tid == 0) {
+    for (int s = 0; s < G::RAW_STAGES; ++s) {
+      s2r_mbar_init(&full[s], 1);
+      s2r_mbar_init(&empty[s], G::NCW);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  __syncthreads();
+  if (warp == G::NCW) {  // producer
+    int it = 0;
+    for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
+      const int s = it % G::RAW_STAGES, n = it / G::RAW_STAGES;
+      if (n > 0) s2r_mbar_wait(&empty[s], (n - 1) & 1);
+      const int ty = (int)(tile / a.tiles_x);
+      const int tx = (int)(tile - (int64_t)ty * a.tiles_x);
+      const double* src = a.src.p + (int64_t)(ty * G::BM - G::R) * a.src.s1 + (tx * G::BN - G::R - G::ODD);
+      s2r_issue_rows(src, a.src.s1, raw + s * G::RAW, G::RR, G::TPR, &full[s], lane);
+    }
+    return;
+  }
   double wa[G::KS], wb[G::KS];
 #pragma unroll
   for (int s = 0; s < G::KS; ++s) {
@@ -59,34 +118,43 @@ __global__ void __launch_bounds__(128, 3) k_s2r2d(S2RArgs a) {
   }
   const int g = lane >> 2, t = lane & 3;
   const bool v0 = 2 * t < G::SW, v1 = 2 * t + 1 < G::SW;
-  for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x) {
+  int it = 0;
+  for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
+    const int s = it % G::RAW_STAGES;
     const int ty = (int)(tile / a.tiles_x);
     const int tx = (int)(tile - (int64_t)ty * a.tiles_x);
-    const double* base = a.src.p + (int64_t)(ty * G::BM - G::R) * a.src.s1 + (tx * G::BN - G::R);
-    __syncthreads();  // the previous tile's fragment reads are done
-#pragma unroll 7
-    for (int e = tid; e < G::NE; e += G::NT) {
-      const int2 l = sL[e];
-      const double v = __ldg(base + l.x);
-      sA[l.y & 0xffff] = v;
-      sB[((unsigned)l.y) >> 16] = v;
+    s2r_mbar_wait(&full[s], (it / G::RAW_STAGES) & 1);
+    asm volatile("bar.sync 1, %0;\n" ::"r"(NC) : "memory");  // previous tile's A/B reads done
+    // implicit stencil2row: scatter the staged region through the LUT (branch-free)
+    const double* rs = raw + s * G::RAW + G::ODD;
+    for (int x = warp; x < G::RR; x += G::NCW) {
+      const double* rrow = rs + x * G::TPR;
+      const uint32_t* lrow = sL + x * G::RC;
+      for (int y = lane; y < G::RC; y += 32) {
+        const double v = rrow[y];
+        const uint32_t l = lrow[y];
+        sA[l & 0xffffu] = v;
+        sB[l >> 16] = v;
+      }
     }
-    __syncthreads();
+    __syncwarp();
+    if (lane == 0) s2r_mbar_arrive(&empty[s]);  // raw stage consumed
+    asm volatile("bar.sync 1, %0;\n" ::"r"(NC) : "memory");  // A/B complete
     const int64_t col = (int64_t)tx * G::BN + g * G::SW + 2 * t;
 #pragma unroll 1
-    for (int xr = warp * (G::BM / 4); xr < (warp + 1) * (G::BM / 4); xr += 2) {
+    for (int xr = warp * (G::BM / G::NCW); xr < (warp + 1) * (G::BM / G::NCW); xr += 2) {
       const double* pa = sA + g * G::PITCH + G::NKV * xr + t;
       const double* pb = sB + g * G::PITCH + G::NKV * xr + t;
       double c00 = 0.0, c01 = 0.0, c10 = 0.0, c11 = 0.0;
 #pragma unroll
-      for (int s = 0; s < G::KS; ++s) {
-        dmma(c00, c01, pa[4 * s], wa[s]);
-        dmma(c10, c11, pa[4 * s + G::NKV], wa[s]);
+      for (int s2 = 0; s2 < G::KS; ++s2) {
+        dmma(c00, c01, pa[4 * s2], wa[s2]);
+        dmma(c10, c11, pa[4 * s2 + G::NKV], wa[s2]);
       }
 #pragma unroll
-      for (int s = 0; s < G::KS; ++s) {
-        dmma(c00, c01, pb[4 * s], wb[s]);
-        dmma(c10, c11, pb[4 * s + G::NKV], wb[s]);
+      for (int s2 = 0; s2 < G::KS; ++s2) {
+        dmma(c00, c01, pb[4 * s2], wb[s2]);
+        dmma(c10, c11, pb[4 * s2 + G::NKV], wb[s2]);
       }
       const int64_t row = (int64_t)ty * G::BM + xr;
       if (row < a.E1) store_pair(a.dst.p + row * a.dst.s1, col, a.E2, v0, v1, c00, c01);
@@ -273,19 +341,18 @@ int num_sms() {
 }
 
 template <class K>
-static cudaError_t launch_persistent(K kernel, int smem, int per_sm, int64_t items, cudaStream_t st,
+static cudaError_t launch_persistent(K kernel, int smem, int nthreads, int64_t items, cudaStream_t st,
                                      const S2RArgs& a) {
   cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return e;
   int occ = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, 128, smem);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, nthreads, smem);
   if (e != cudaSuccess) return e;
   if (occ < 1) return cudaErrorInvalidConfiguration;
-  (void)per_sm;
   int64_t grid = (int64_t)occ * num_sms();
   if (grid > items) grid = items;
   if (grid < 1) grid = 1;
-  kernel<<<(unsigned)grid, 128, smem, st>>>(a);
+  kernel<<<(unsigned)grid, nthreads, smem, st>>>(a);
   return cudaGetLastError();
 }
 
@@ -319,19 +386,19 @@ cudaError_t launch_s2r(int ndim, int nk, int nf, const S2RArgs& a, int tc_mask, 
   if (smem < 0) return cudaErrorInvalidValue;
   if (ndim == 1) {
     switch (nk) {
-      case 3: return launch_persistent(k_s2r1d<3>, smem, 4, a.ntiles, st, a);
-      case 5: return launch_persistent(k_s2r1d<5>, smem, 4, a.ntiles, st, a);
-      case 7: return launch_persistent(k_s2r1d<7>, smem, 4, a.ntiles, st, a);
-      case 9: return launch_persistent(k_s2r1d<9>, smem, 4, a.ntiles, st, a);
-      case 11: return launch_persistent(k_s2r1d<11>, smem, 4, a.ntiles, st, a);
-      case 13: return launch_persistent(k_s2r1d<13>, smem, 4, a.ntiles, st, a);
-      case 15: return launch_persistent(k_s2r1d<15>, smem, 4, a.ntiles, st, a);
+      case 3: return launch_persistent(k_s2r1d<3>, smem, 128, a.ntiles, st, a);
+      case 5: return launch_persistent(k_s2r1d<5>, smem, 128, a.ntiles, st, a);
+      case 7: return launch_persistent(k_s2r1d<7>, smem, 128, a.ntiles, st, a);
+      case 9: return launch_persistent(k_s2r1d<9>, smem, 128, a.ntiles, st, a);
+      case 11: return launch_persistent(k_s2r1d<11>, smem, 128, a.ntiles, st, a);
+      case 13: return launch_persistent(k_s2r1d<13>, smem, 128, a.ntiles, st, a);
+      case 15: return launch_persistent(k_s2r1d<15>, smem, 128, a.ntiles, st, a);
     }
   } else if (ndim == 2) {
     switch (nk) {
-      case 3: return launch_persistent(k_s2r2d<3>, smem, 3, a.ntiles, st, a);
-      case 5: return launch_persistent(k_s2r2d<5>, smem, 3, a.ntiles, st, a);
-      case 7: return launch_persistent(k_s2r2d<7>, smem, 3, a.ntiles, st, a);
+      case 3: return launch_persistent(k_s2r2d<3>, smem, S2R2D<3>::NT, a.ntiles, st, a);
+      case 5: return launch_persistent(k_s2r2d<5>, smem, S2R2D<5>::NT, a.ntiles, st, a);
+      case 7: return launch_persistent(k_s2r2d<7>, smem, S2R2D<7>::NT, a.ntiles, st, a);
     }
   } else if (nk == 3) {
     auto kern = k_s2r3d<3>;

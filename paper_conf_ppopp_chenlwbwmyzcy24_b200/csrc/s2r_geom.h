@@ -26,8 +26,16 @@ struct S2R2D {
   static constexpr int STRIPS = 8;             // stencil2row rows per CTA (+1 dirty row)
   static constexpr int PITCH = s2r_pitch(NK * RR);
   static constexpr int R = (NK - 1) / 2;
-  static constexpr int NT = 128;
-  static constexpr int SMEM = 2 * (STRIPS + 1) * PITCH * 8 + NE * 8;
+  // B200 staging: the raw input region arrives by cp.async.bulk rows (16-B aligned, hence the
+  // ODD shift) in a 2-stage ring filled by one producer warp; 8 consumer warps scatter it
+  // through the LUT into A/B and run the dual tessellations (4 output rows each).
+  static constexpr int ODD = R & 1;
+  static constexpr int TPR = (ODD + RC + 1) / 2 * 2;  // raw staged row length (even)
+  static constexpr int RAW = RR * TPR;                 // doubles per raw stage
+  static constexpr int RAW_STAGES = 2;
+  static constexpr int NCW = 8;                        // consumer warps
+  static constexpr int NT = 32 * (NCW + 1);
+  static constexpr int SMEM = 2 * (STRIPS + 1) * PITCH * 8 + NE * 4 + RAW_STAGES * RAW * 8;
 };
 
 template <int NK>

@@ -177,3 +177,26 @@ def test_full_size_sampled(csx, name, ext, T):
     ref = oracle.sample(u0, w, "fixed", T, pts)
     vals = np.array([got[p] for p in pts])
     assert np.max(np.abs(vals - ref)) / np.max(np.abs(got)) <= TOL, info
+
+
+@pytest.mark.parametrize("name", ["heat3d", "box3d27p"])
+@pytest.mark.parametrize("engine", ["tc_tile", "tc_s2r"])
+def test_parity_3d_zchunks(csx, name, engine):
+    """3D grids spanning several z chunks (ragged last chunk) and ragged (y, x) tiles."""
+    s = synth.SHAPES[name]
+    u0 = synth.grid((70, 37, 45), seed=31)
+    w = synth.random_weights(name)
+    for bc in ("fixed", "periodic"):
+        got, info = run_gpu(csx, u0, w, s.kind, bc, 4, engine=engine)
+        assert info["engine_name"] == engine
+        assert rel(got, oracle.run(u0, w, bc, 4)) <= TOL, (name, engine, bc)
+
+
+def test_direct_comparator_2d_all_radii(csx):
+    """The 2D CUDA-core comparator (k_direct2d) for r = 1..3 and its temporal-blocking depths."""
+    for ndim, r, tf in [(2, 1, 1), (2, 1, 2), (2, 1, 3), (2, 2, 1), (2, 3, 1)]:
+        w = synth.random_signed_weights(ndim, r, seed=40 + r)
+        u0 = synth.grid((131, 150), seed=41)
+        for bc in ("fixed", "periodic"):
+            got, info = run_gpu(csx, u0, w, "box", bc, 9, engine="direct", fuse_steps=tf)
+            assert rel(got, oracle.run(u0, w, bc, 9)) <= TOL, (r, tf, bc)
