@@ -133,12 +133,24 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
       a.frags = ps.d_tile_frags;
       if (p->ndim == 3)
         for (int dz = 0; dz < ps.nk; ++dz) a.tc_mask |= ps.plane_is_tc[dz] << dz;
-      if (p->bc == CSX_BC_FIXED && p->ndim == 2) {  // band fix-up fused into the edge CTAs
+      if (p->bc == CSX_BC_FIXED && p->ndim == 1) {  // 1D band recomputed in-kernel
         a.fix_band = p->radius * ps.tf;
         a.r = p->radius;
         a.wbase = p->d_wbase;
+        a.gorg2 = c.gorg[2];
+        a.GE2 = p->E[2];
+      }
+      if (p->bc == CSX_BC_FIXED && p->ndim >= 2) {
+        // 2D: the edge CTAs leave the band to k_band (Tf > 1) or write the held frame (Tf = 1);
+        // 3D (Tf = 1): the frame is written from the staged plane
+        a.fix_band = p->radius * ps.tf;
+        a.hold_frame = ps.tf == 1;
+        a.r = p->radius;
+        a.wbase = p->d_wbase;
+        a.gorg0 = c.gorg[0];
         a.gorg1 = c.gorg[1];
         a.gorg2 = c.gorg[2];
+        a.GE0 = p->E[0];
         a.GE1 = p->E[1];
         a.GE2 = p->E[2];
       }
@@ -196,7 +208,8 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
       e = launch_direct(d, st);
     if (e != cudaSuccess) return cuda_fail(e, "direct launch");
     p->n_launches += 1;
-  } else if (p->bc == CSX_BC_FIXED) {
+  } else if (p->bc == CSX_BC_FIXED && !(eng == CSX_ENGINE_TC_TILE && p->ndim == 1) &&
+             !(eng == CSX_ENGINE_TC_TILE && p->ndim >= 2 && ps.tf == 1)) {  // else done in-kernel
     if (ps.tf == 1 || p->ndim == 3) {
       // the composed window is the plain stencil: only the held frame needs restoring
       e = launch_frame_copy(c.src, c.dst, c.E, c.gorg, p->E, real, p->radius, st);

@@ -28,10 +28,11 @@ struct S2RArgs {
   // fix_band = r*Tf of a GLOBAL face by Tf plain steps on CUDA cores from the staged tile.
   int tc_mask = 0;                // 3D: bit dz set = z offset dz runs on tensor cores
   int fix_band = 0;
+  int hold_frame = 0;             // write held (frame) values from the staged tile (Tf = 1)
   int r = 0;
   const double* wbase = nullptr;  // base weights (2r+1)^2
-  int64_t gorg1 = 0, gorg2 = 0;   // local origin in global coordinates
-  int64_t GE1 = 0, GE2 = 0;       // global extents
+  int64_t gorg0 = 0, gorg1 = 0, gorg2 = 0;  // local origin in global coordinates
+  int64_t GE0 = 0, GE1 = 0, GE2 = 0;        // global extents
 };
 
 struct DirectArgs {

@@ -163,34 +163,56 @@ cudaError_t launch_direct(const DirectArgs& a, cudaStream_t st) {
 }
 
 // ------------------------------------------------------------------------------------------
+// FIXED frame copy, one thread per frame element.  Local rows (z, y) are either entirely in
+// the global frame (a frame plane or frame row: all E2 columns copied) or contribute only their
+// 2r frame columns.  Work = O(frame size), not O(grid).
 __global__ void k_frame_copy(CView src, View dst, int64_t E0, int64_t E1, int64_t E2, int64_t g0,
                              int64_t g1, int64_t g2, int64_t G0, int64_t G1, int64_t G2, int real0,
                              int real1, int r) {
+  // local index ranges of the frame rows / planes
   const int64_t nrows = E0 * E1;
-  for (int64_t row = blockIdx.x; row < nrows; row += gridDim.x) {
+  const int64_t total = nrows * 2 * r;  // column part for every row (frame rows re-copy: harmless)
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t row = i / (2 * r);
+    const int k = (int)(i - row * 2 * r);
     const int64_t z = row / E1, y = row - z * E1;
-    const int64_t gz = g0 + z, gy = g1 + y;
-    const bool whole = (real0 && (gz < r || gz >= G0 - r)) || (real1 && (gy < r || gy >= G1 - r));
-    const double* s = src.p + z * src.s0 + y * src.s1;
-    double* d = dst.p + z * dst.s0 + y * dst.s1;
-    if (whole) {
-      for (int64_t x = threadIdx.x; x < E2; x += blockDim.x) d[x] = s[x];
+    const int64_t gx = k < r ? k : G2 - 2 * r + k;
+    const int64_t x = gx - g2;
+    if (x >= 0 && x < E2) dst.p[z * dst.s0 + y * dst.s1 + x] = src.p[z * src.s0 + y * src.s1 + x];
+  }
+  // full frame rows: rows whose plane or row index is in the global frame
+  const int64_t nfr_y = real1 ? 2 * r : 0;           // frame rows per plane
+  const int64_t nfr_z = real0 ? 2 * r : 0;           // frame planes
+  const int64_t rows_a = nfr_z * E1;                 // rows of the frame planes
+  const int64_t rows_b = (real1 ? E0 : 0) * nfr_y;   // frame rows of every plane
+  const int64_t total2 = (rows_a + rows_b) * E2;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total2;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t rr = i / E2, x = i - rr * E2;
+    int64_t z, y;
+    if (rr < rows_a) {
+      const int64_t kz = rr / E1;
+      y = rr - kz * E1;
+      const int64_t gz = kz < r ? kz : G0 - 2 * r + kz;
+      z = gz - g0;
+      if (z < 0 || z >= E0) continue;
     } else {
-      for (int64_t k = threadIdx.x; k < 2 * r; k += blockDim.x) {
-        const int64_t gx = k < r ? k : G2 - 2 * r + k;  // global frame column
-        const int64_t x = gx - g2;
-        if (x >= 0 && x < E2) d[x] = s[x];
-      }
+      const int64_t q = rr - rows_a;
+      z = q / nfr_y;
+      const int64_t ky = q - z * nfr_y;
+      const int64_t gy = ky < r ? ky : G1 - 2 * r + ky;
+      y = gy - g1;
+      if (y < 0 || y >= E1) continue;
     }
+    dst.p[z * dst.s0 + y * dst.s1 + x] = src.p[z * src.s0 + y * src.s1 + x];
   }
 }
 
 cudaError_t launch_frame_copy(CView src, View dst, const int64_t* E, const int64_t* gorg,
                               const int64_t* GE, const int* real, int r, cudaStream_t st) {
-  const int64_t nrows = E[0] * E[1];
-  const int64_t grid = nrows < 8 * num_sms() ? nrows : 8 * num_sms();
-  k_frame_copy<<<(unsigned)grid, 128, 0, st>>>(src, dst, E[0], E[1], E[2], gorg[0], gorg[1], gorg[2],
-                                               GE[0], GE[1], GE[2], real[0], real[1], r);
+  k_frame_copy<<<4 * num_sms(), 256, 0, st>>>(src, dst, E[0], E[1], E[2], gorg[0], gorg[1], gorg[2],
+                                             GE[0], GE[1], GE[2], real[0], real[1], r);
   return cudaGetLastError();
 }
 
@@ -204,10 +226,25 @@ __global__ void k_pack(const double* __restrict__ in, View dst, int64_t E1, int6
   }
 }
 
+// few long rows (1D): one thread per element
+__global__ void k_pack_flat(const double* __restrict__ in, View dst, int64_t E1, int64_t E2,
+                            int64_t n) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t row = i / E2, x = i - row * E2;
+    const int64_t z = row / E1, y = row - z * E1;
+    dst.p[z * dst.s0 + y * dst.s1 + x] = in[i];
+  }
+}
+
 cudaError_t launch_pack(const double* in, View dst, const int64_t* E, cudaStream_t st) {
   const int64_t nrows = E[0] * E[1];
-  int64_t grid = nrows < 65535 ? nrows : 65535;
-  k_pack<<<(unsigned)grid, 256, 0, st>>>(in, dst, E[1], E[2], nrows);
+  if (nrows < 4 * num_sms()) {
+    k_pack_flat<<<8 * num_sms(), 256, 0, st>>>(in, dst, E[1], E[2], nrows * E[2]);
+  } else {
+    const int64_t grid = nrows < 65535 ? nrows : 65535;
+    k_pack<<<(unsigned)grid, 256, 0, st>>>(in, dst, E[1], E[2], nrows);
+  }
   return cudaGetLastError();
 }
 

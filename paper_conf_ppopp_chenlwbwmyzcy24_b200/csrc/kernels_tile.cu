@@ -67,17 +67,25 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(bar)) : "memory");
 }
 
+constexpr int s2r_pitch_dev(int min_pitch) {
+  int p = min_pitch;
+  while (p % 16 != 4 && p % 16 != 12) ++p;
+  return p;
+}
+
 // Compile-time geometry of one TC_TILE instantiation.
-template <int NK_, int A_, int B_, int KC_, int G_, int WM_, int WN_, int STAGES_>
+template <int NK_, int A_, int B_, int KC_, int G_, int WM_, int WN_, int STAGES_, int CG_ = 1>
 struct TileCfg {
   static constexpr int NK = NK_, A = A_, B = B_, KC = KC_, G = G_, WM = WM_, WN = WN_;
   static constexpr int STAGES = STAGES_;
+  static constexpr int CG = CG_;                    // 8-block column groups per warp
   static constexpr int R = (NK - 1) / 2;
   static constexpr int ODD = R & 1;                 // smem col = region col + ODD (16-B aligned rows)
   static constexpr int KR = A + NK - 1;             // input rows per output block
   static constexpr int KS = KR * KC / 4;            // k-slices (DMMAs) per output block
   static constexpr int BM = WM * A * G;             // CTA output rows
-  static constexpr int BN = WN * 8 * B;             // CTA output cols
+  static constexpr int WC = CG * 8 * B;             // output cols per warp
+  static constexpr int BN = WN * WC;                // CTA output cols
   static constexpr int RR = BM + NK - 1;            // staged input rows
   static constexpr int TP = ((ODD + BN + KC - B) + 1) / 2 * 2;  // staged row length (even)
   static constexpr int STAGE = RR * TP;             // doubles per stage
@@ -146,71 +154,98 @@ __global__ void __launch_bounds__(C::NT, 1) k_tile2d(S2RArgs a) {
     mbar_wait(&full[s], (it / C::STAGES) & 1);
     const int ty = (int)(tile / a.tiles_x);
     const int tx = (int)(tile - (int64_t)ty * a.tiles_x);
-    const double* base = smem + s * C::STAGE + (wm * C::A * C::G) * C::TP + wn * 8 * C::B + C::ODD +
+    const double* base = smem + s * C::STAGE + (wm * C::A * C::G) * C::TP + wn * C::WC + C::ODD +
                          C::B * g + t;
-    double acc[C::G][2];
+    double acc[C::CG][C::G][2];
 #pragma unroll
-    for (int j = 0; j < C::G; ++j) acc[j][0] = acc[j][1] = 0.0;
+    for (int cg = 0; cg < C::CG; ++cg)
+#pragma unroll
+      for (int j = 0; j < C::G; ++j) acc[cg][j][0] = acc[cg][j][1] = 0.0;
     // Stream the warp's input rows; each A fragment (4 cells of one row) feeds every output
     // block whose window contains the row.  Consecutive DMMAs go to different accumulators.
 #pragma unroll
     for (int ra = 0; ra < C::A * C::G + C::NK - 1; ++ra) {
-      double f[C::KC / 4];
+      double f[C::CG][C::KC / 4];
 #pragma unroll
-      for (int h = 0; h < C::KC / 4; ++h) f[h] = base[ra * C::TP + 4 * h];
+      for (int cg = 0; cg < C::CG; ++cg)
+#pragma unroll
+        for (int h = 0; h < C::KC / 4; ++h) f[cg][h] = base[ra * C::TP + cg * 8 * C::B + 4 * h];
 #pragma unroll
       for (int h = 0; h < C::KC / 4; ++h)
 #pragma unroll
         for (int j = 0; j < C::G; ++j) {
           const int rho = ra - C::A * j;
-          if (rho >= 0 && rho < C::KR) dmma_t(acc[j][0], acc[j][1], f[h], wf[rho * (C::KC / 4) + h]);
+          if (rho >= 0 && rho < C::KR)
+#pragma unroll
+            for (int cg = 0; cg < C::CG; ++cg)
+              dmma_t(acc[cg][j][0], acc[cg][j][1], f[cg][h], wf[rho * (C::KC / 4) + h]);
         }
     }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&empty[s]);  // this warp no longer reads stage s
-    // FIXED: band outputs of an edge tile are written by k_band (kernels_band.cu)
+    // FIXED: band outputs of an edge tile are written by k_band (kernels_band.cu) after a pass
+    // of Tf > 1 steps; for Tf = 1 the band is the held frame, written here from the staged tile.
     const bool edge = tile_is_edge<C>(a, ty, tx);
-    // store: block j covers output rows ty*BM + wm*A*G + A*j + [0, A), cols tx*BN + wn*8B + B*g + [0, B)
-    const int64_t col = (int64_t)tx * C::BN + wn * 8 * C::B + C::B * g + beta;
+    if (!edge) {
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[s]);  // this warp no longer reads stage s
+    }
+    // store: block j of column group cg covers output rows ty*BM + wm*A*G + A*j + [0, A),
+    // cols tx*BN + wn*WC + cg*8B + B*g + [0, B)
     const int64_t row0 = (int64_t)ty * C::BM + wm * C::A * C::G + alpha;
-    const int64_t gcol = col + a.gorg2;
-    const bool col_band = edge && (gcol < a.fix_band || gcol + 1 >= a.GE2 - a.fix_band);
 #pragma unroll
-    for (int j = 0; j < C::G; ++j) {
-      const int64_t row = row0 + C::A * j;
-      const int64_t grow = row + a.gorg1;
-      if (edge && (col_band || grow < a.fix_band || grow >= a.GE1 - a.fix_band)) {
-        // band points were written by band_fix; only a pair straddling the band edge keeps
-        // its non-band half
-        if (!(col_band && !(grow < a.fix_band || grow >= a.GE1 - a.fix_band))) continue;
-        if (row >= a.E1) continue;
-        double* p = a.dst.p + row * a.dst.s1 + col;
-        if (gcol >= a.fix_band && gcol < a.GE2 - a.fix_band && col < a.E2) p[0] = acc[j][0];
-        if (gcol + 1 >= a.fix_band && gcol + 1 < a.GE2 - a.fix_band && col + 1 < a.E2) p[1] = acc[j][1];
-        continue;
-      }
-      if (row < a.E1 && col < a.E2) {
-        double* p = a.dst.p + row * a.dst.s1 + col;
-        if (col + 1 < a.E2 && ((reinterpret_cast<uintptr_t>(p) & 15) == 0)) {
-          *reinterpret_cast<double2*>(p) = make_double2(acc[j][0], acc[j][1]);
-        } else {
-          p[0] = acc[j][0];
-          if (col + 1 < a.E2) p[1] = acc[j][1];
+    for (int cg = 0; cg < C::CG; ++cg) {
+      const int64_t col = (int64_t)tx * C::BN + wn * C::WC + cg * 8 * C::B + C::B * g + beta;
+#pragma unroll
+      for (int j = 0; j < C::G; ++j) {
+        const int64_t row = row0 + C::A * j;
+        if (!edge) {
+          if (row < a.E1 && col < a.E2) {
+            double* p = a.dst.p + row * a.dst.s1 + col;
+            if (col + 1 < a.E2 && ((reinterpret_cast<uintptr_t>(p) & 15) == 0)) {
+              *reinterpret_cast<double2*>(p) = make_double2(acc[cg][j][0], acc[cg][j][1]);
+            } else {
+              p[0] = acc[cg][j][0];
+              if (col + 1 < a.E2) p[1] = acc[cg][j][1];
+            }
+          }
+        } else if (row < a.E1) {
+          const int64_t grow = row + a.gorg1;
+          const bool rowband = grow < a.fix_band || grow >= a.GE1 - a.fix_band;
+#pragma unroll
+          for (int e = 0; e < 2; ++e) {
+            const int64_t c = col + e;
+            if (c >= a.E2) continue;
+            const int64_t gc = c + a.gorg2;
+            double v = acc[cg][j][e];
+            if (rowband || gc < a.fix_band || gc >= a.GE2 - a.fix_band) {
+              if (!a.hold_frame) continue;
+              v = smem[s * C::STAGE + (int)(row - (int64_t)ty * C::BM + C::R) * C::TP +
+                       (int)(c - (int64_t)tx * C::BN) + C::R + C::ODD];
+            }
+            a.dst.p[row * a.dst.s1 + c] = v;
+          }
         }
       }
+    }
+    if (edge) {
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[s]);
     }
   }
 }
 
 // nk -> (a, b, kc); G blocks per warp column, WM x WN consumer warps, STAGES-deep ring.
 // Variant 0: 12 DMMA warps, 3 stages (CTA 96 x 64).  Variant 1: 16 DMMA warps, 2 stages
-// (CTA 128 x 64).  CSX_TILE_VARIANT selects (default 0).
+// (CTA 128 x 64).  Variant 2: 12 warps of 2 column groups x 4 block rows (CTA 96 x 64) — twice
+// the independent accumulator chains per input row.  CSX_TILE_VARIANT selects (default 0).
 using Tile3 = TileCfg<3, 4, 2, 4, 8, 3, 4, 3>;
 using Tile5 = TileCfg<5, 2, 4, 8, 8, 6, 2, 3>;
 using Tile7 = TileCfg<7, 4, 2, 8, 8, 3, 4, 3>;
 using Tile3b = TileCfg<3, 4, 2, 4, 8, 4, 4, 2>;
 using Tile5b = TileCfg<5, 2, 4, 8, 8, 8, 2, 2>;
 using Tile7b = TileCfg<7, 4, 2, 8, 8, 4, 4, 2>;
+using Tile3c = TileCfg<3, 4, 2, 4, 4, 6, 2, 3, 2>;
+using Tile5c = TileCfg<5, 2, 4, 8, 4, 12, 1, 3, 2>;
+using Tile7c = TileCfg<7, 4, 2, 8, 4, 6, 2, 3, 2>;
 
 static int tile_variant() {
   static int v = -1;
@@ -347,22 +382,44 @@ __global__ void __launch_bounds__(C::NT, 2) k_tile3d(S2RArgs a, int tc_mask) {
           }
         }
       }
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&empty[(q0 + (zo - z0)) % C::STAGES]);  // plane zo-R is done
+      // FIXED frame (held points) of this output plane: the staged plane zo (dz = R) holds them
+      const int64_t gzo = zo + a.gorg0;
+      const bool plane_frame = a.hold_frame && (gzo < C::R || gzo >= a.GE0 - C::R);
+      const bool edge = a.hold_frame &&
+                        (plane_frame || (int64_t)ty * C::BM + a.gorg1 < C::R ||
+                         (int64_t)(ty + 1) * C::BM + a.gorg1 > a.GE1 - C::R ||
+                         (int64_t)tx * C::BN + a.gorg2 < C::R || (int64_t)(tx + 1) * C::BN + a.gorg2 > a.GE2 - C::R);
+      const double* cstg = smem + ((q0 + (zo - z0) + C::R) % C::STAGES) * C::STAGE;
       double* plane = a.dst.p + zo * a.dst.s0;
 #pragma unroll
       for (int j = 0; j < C::G; ++j) {
         const int64_t row = row0 + C::A * j;
         if (row < a.E1 && col < a.E2) {
           double* p = plane + row * a.dst.s1 + col;
-          if (col + 1 < a.E2 && ((reinterpret_cast<uintptr_t>(p) & 15) == 0)) {
-            *reinterpret_cast<double2*>(p) = make_double2(acc[j][0], acc[j][1]);
+          if (!edge) {
+            if (col + 1 < a.E2 && ((reinterpret_cast<uintptr_t>(p) & 15) == 0)) {
+              *reinterpret_cast<double2*>(p) = make_double2(acc[j][0], acc[j][1]);
+            } else {
+              p[0] = acc[j][0];
+              if (col + 1 < a.E2) p[1] = acc[j][1];
+            }
           } else {
-            p[0] = acc[j][0];
-            if (col + 1 < a.E2) p[1] = acc[j][1];
+            const int64_t grow = row + a.gorg1;
+            const bool rf = plane_frame || grow < C::R || grow >= a.GE1 - C::R;
+#pragma unroll
+            for (int e = 0; e < 2; ++e) {
+              const int64_t c = col + e, gc = c + a.gorg2;
+              if (c >= a.E2) continue;
+              double v = acc[j][e];
+              if (rf || gc < C::R || gc >= a.GE2 - C::R)
+                v = cstg[(int)(row - (int64_t)ty * C::BM + C::R) * C::TP + (int)(c - (int64_t)tx * C::BN) + C::R + C::ODD];
+              p[e] = v;
+            }
           }
         }
       }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[(q0 + (zo - z0)) % C::STAGES]);  // plane zo-R is done
     }
     // release the last 2R planes of the item (not released by an output plane)
     __syncwarp();
@@ -375,8 +432,197 @@ __global__ void __launch_bounds__(C::NT, 2) k_tile3d(S2RArgs a, int tc_mask) {
 using Tile3D3 = Tile3DCfg<3, 8, 2, 2, 4, 32>;  // CTA 64 x 32 outputs, 4-plane ring, 32 planes per item
 
 
+// ------------------------------------------------------------------------------------------
+// 1D (P.1779-1786) on the TC_TILE pipeline.  The paper's 1D dual tessellation is kept exactly —
+// strip k of a segment holds outputs [k(nk+1), (k+1)(nk+1)), Tile_A row = the nk inputs of the
+// strip, Tile_B row = the next nk, W_A / W_B as in 2D, N fragments for nk+1 > 8 (reading A7) —
+// but the 8 M rows of a DMMA are 8 different SEGMENTS of the tile, staged by cp.async.bulk with
+// a segment pitch P = 4 or 12 (mod 16) doubles.  The A/B fragments are then strided views of
+// the staged input (conflict-free, no LUT scatter), and the kernel streams HBM through a
+// STAGES-deep ring (the 1D path is HBM-bound: 16/Tf bytes per point-step).
+template <int NK_, int L_, int NCW_, int STAGES_>
+struct Tile1DCfg {
+  static constexpr int NK = NK_, L = L_, NCW = NCW_, STAGES = STAGES_;
+  static constexpr int SW = NK + 1;
+  static constexpr int NF = (SW + 7) / 8;
+  static constexpr int KA = (NK + 3) / 4;
+  static constexpr int R = (NK - 1) / 2;
+  static constexpr int ODD = R & 1;
+  static constexpr int SL = ((ODD + L + NK + 4 * KA) + 1) / 2 * 2;  // staged segment length
+  static constexpr int P = s2r_pitch_dev(SL);                        // segment pitch (doubles)
+  static constexpr int STAGE = 8 * P;
+  static constexpr int TILE = 8 * L;                                 // outputs per tile
+  static constexpr int NT = 32 * (NCW + 1);
+  static constexpr int SMEM = STAGES * STAGE * 8;
+  static_assert(L % SW == 0, "segment length must be a multiple of nk+1");
+};
+
+template <class C>
+__global__ void __launch_bounds__(C::NT, 2) k_tile1d(S2RArgs a) {
+  extern __shared__ __align__(128) double smem[];
+  __shared__ __align__(8) uint64_t full[C::STAGES], empty[C::STAGES];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  if (tid == 0) {
+    for (int s = 0; s < C::STAGES; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], C::NCW);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  __syncthreads();
+  if (warp == C::NCW) {  // producer: 8 segment copies per tile
+    int it = 0;
+    for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
+      const int s = it % C::STAGES, n = it / C::STAGES;
+      if (n > 0) mbar_wait(&empty[s], (n - 1) & 1);
+      const int64_t t0 = tile * C::TILE;
+      int nseg = (int)min((int64_t)8, (a.E2 - t0 + C::L - 1) / C::L);
+      if (lane == 0) mbar_expect_tx(&full[s], (uint32_t)(nseg * C::SL * 8));
+      __syncwarp();
+      if (lane < nseg) {
+        const double* src = a.src.p + t0 + (int64_t)lane * C::L - C::R - C::ODD;
+        bulk_g2s(smem + s * C::STAGE + lane * C::P, src, (uint32_t)(C::SL * 8), &full[s]);
+      }
+    }
+    return;
+  }
+  const int g = lane >> 2, t = lane & 3;
+  double wa[C::NF][C::KA], wb[C::NF][C::KA];
+#pragma unroll
+  for (int f = 0; f < C::NF; ++f)
+#pragma unroll
+    for (int s = 0; s < C::KA; ++s) {
+      wa[f][s] = a.frags[((0 * C::NF + f) * C::KA + s) * 32 + lane];
+      wb[f][s] = a.frags[((1 * C::NF + f) * C::KA + s) * 32 + lane];
+    }
+  int it = 0;
+  for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
+    const int s = it % C::STAGES;
+    mbar_wait(&full[s], (it / C::STAGES) & 1);
+    const double* seg = smem + s * C::STAGE + g * C::P + C::ODD + t;  // this lane's segment g
+    const int64_t t0 = tile * C::TILE + (int64_t)g * C::L;
+    constexpr int NSTRIP = C::L / C::SW;
+    double res[(NSTRIP + C::NCW - 1) / C::NCW][C::NF][2];
+#pragma unroll
+    for (int q = 0; q < (NSTRIP + C::NCW - 1) / C::NCW; ++q) {
+      const int k = warp + q * C::NCW;
+      if (k < NSTRIP) {
+#pragma unroll
+        for (int f = 0; f < C::NF; ++f) res[q][f][0] = res[q][f][1] = 0.0;
+#pragma unroll
+        for (int s2 = 0; s2 < C::KA; ++s2) {
+          const double xa = seg[k * C::SW + 4 * s2];
+          const double xb = seg[k * C::SW + C::NK + 4 * s2];
+#pragma unroll
+          for (int f = 0; f < C::NF; ++f) {
+            dmma_t(res[q][f][0], res[q][f][1], xa, wa[f][s2]);
+            dmma_t(res[q][f][0], res[q][f][1], xb, wb[f][s2]);
+          }
+        }
+      }
+    }
+    // FIXED: the band b = r*Tf at each global end is recomputed by Tf plain steps (reading A1)
+    // by warp 0 from the staged segments, one lane per point, neighbours via shuffles.
+    const int fb = a.fix_band;
+    const int64_t tg0 = tile * C::TILE + a.gorg2;  // global index of the tile's first output
+    if (fb > 0 && warp == 0 && (tg0 < fb || tg0 + C::TILE > a.GE2 - fb)) {
+      const int r = a.r, tf = fb / r, D = r * (tf - 1);
+      for (int sg = 0; sg < 8; ++sg) {
+        const int64_t s0 = tg0 + (int64_t)sg * C::L;  // global range of segment sg
+        for (int side = 0; side < 2; ++side) {
+          int64_t q0 = side == 0 ? 0 : a.GE2 - fb, q1 = side == 0 ? fb : a.GE2;
+          q0 = max(q0, s0);
+          q1 = min(q1, min(s0 + (int64_t)C::L, a.GE2));
+          q1 = min(q1, a.gorg2 + a.E2);
+          if (q0 >= q1) continue;
+          // lane l <-> global position q0 - D + l; level 0 from the staged segment
+          const int64_t gp = q0 - D + lane;
+          const double* sgm = smem + s * C::STAGE + sg * C::P + C::ODD;  // staged: index = pos - s0 + R
+          const bool hold = gp < r || gp >= a.GE2 - r;
+          const int li = (int)(gp - s0) + C::R;
+          double v = 0.0;
+          if (li >= 0 && li < C::SL) {
+            if (hold) {
+              v = sgm[li];
+            } else {
+              for (int o = -r; o <= r; ++o) v = fma(__ldg(a.wbase + o + r), sgm[li + o], v);
+            }
+          }
+          for (int lv = 2; lv <= tf; ++lv) {
+            double nv = 0.0;
+            for (int o = -r; o <= r; ++o) {
+              const double x = __shfl_sync(0xffffffffu, v, (lane + o) & 31);
+              nv = fma(__ldg(a.wbase + o + r), x, nv);
+            }
+            v = hold ? v : nv;
+          }
+          const int64_t lp = gp - a.gorg2;  // local position
+          if (gp >= q0 && gp < q1 && lane < 32) a.dst.p[lp] = v;
+        }
+      }
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[s]);
+#pragma unroll
+    for (int q = 0; q < (NSTRIP + C::NCW - 1) / C::NCW; ++q) {
+      const int k = warp + q * C::NCW;
+      if (k < NSTRIP) {
+#pragma unroll
+        for (int f = 0; f < C::NF; ++f) {
+          const int c = 8 * f + 2 * t;
+          const int64_t o = t0 + (int64_t)k * C::SW + c;
+          if (fb > 0) {  // band points are written by the band code above
+            const int64_t go = o + a.gorg2;
+            if (c < C::SW && o < a.E2 && !(go < fb || go >= a.GE2 - fb)) a.dst.p[o] = res[q][f][0];
+            if (c + 1 < C::SW && o + 1 < a.E2 && !(go + 1 < fb || go + 1 >= a.GE2 - fb))
+              a.dst.p[o + 1] = res[q][f][1];
+            continue;
+          }
+          if (c < C::SW && o < a.E2) {
+            double* p = a.dst.p + o;
+            if (c + 1 < C::SW && o + 1 < a.E2 && ((reinterpret_cast<uintptr_t>(p) & 15) == 0)) {
+              *reinterpret_cast<double2*>(p) = make_double2(res[q][f][0], res[q][f][1]);
+            } else {
+              p[0] = res[q][f][0];
+              if (c + 1 < C::SW && o + 1 < a.E2) p[1] = res[q][f][1];
+            }
+          }
+        }
+      }
+    }
+  }
+}
+
+template <class C>
+static cudaError_t launch_tile1d_cfg(S2RArgs a, cudaStream_t st) {
+  a.ntiles = (a.E2 + C::TILE - 1) / C::TILE;
+  cudaError_t e = cudaFuncSetAttribute(k_tile1d<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
+  if (e != cudaSuccess) return e;
+  int occ = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_tile1d<C>, C::NT, C::SMEM);
+  if (e != cudaSuccess) return e;
+  int64_t grid = (int64_t)(occ < 1 ? 1 : occ) * num_sms();
+  if (grid > a.ntiles) grid = a.ntiles;
+  k_tile1d<C><<<(unsigned)grid, C::NT, C::SMEM, st>>>(a);
+  return cudaGetLastError();
+}
+
+static cudaError_t launch_tile1d(int nk, const S2RArgs& a, cudaStream_t st) {
+  switch (nk) {
+    case 3: return launch_tile1d_cfg<Tile1DCfg<3, 256, 4, 6>>(a, st);
+    case 5: return launch_tile1d_cfg<Tile1DCfg<5, 252, 4, 6>>(a, st);
+    case 7: return launch_tile1d_cfg<Tile1DCfg<7, 256, 4, 6>>(a, st);
+    case 9: return launch_tile1d_cfg<Tile1DCfg<9, 250, 4, 6>>(a, st);
+    case 11: return launch_tile1d_cfg<Tile1DCfg<11, 252, 4, 6>>(a, st);
+    case 13: return launch_tile1d_cfg<Tile1DCfg<13, 252, 4, 6>>(a, st);
+    case 15: return launch_tile1d_cfg<Tile1DCfg<15, 256, 4, 6>>(a, st);
+  }
+  return cudaErrorNotSupported;
+}
+
 bool tile_kernel_exists(int ndim, int nk) {
-  return (ndim == 2 && (nk == 3 || nk == 5 || nk == 7)) || (ndim == 3 && nk == 3);
+  return (ndim == 1 && (nk & 1) && nk >= 3 && nk <= 15) ||
+         (ndim == 2 && (nk == 3 || nk == 5 || nk == 7)) || (ndim == 3 && nk == 3);
 }
 
 template <class C>
@@ -412,6 +658,7 @@ static cudaError_t launch_tile3d_cfg(S2RArgs a, int tc_mask, cudaStream_t st) {
 }
 
 cudaError_t launch_tile(int ndim, int nk, const S2RArgs& a, cudaStream_t st) {
+  if (ndim == 1) return launch_tile1d(nk, a, st);
   if (ndim == 3) {
     if (nk == 3) return launch_tile3d_cfg<Tile3D3>(a, a.tc_mask, st);
     return cudaErrorNotSupported;
@@ -419,9 +666,9 @@ cudaError_t launch_tile(int ndim, int nk, const S2RArgs& a, cudaStream_t st) {
   if (ndim != 2) return cudaErrorNotSupported;
   const int v = tile_variant();
   switch (nk) {
-    case 3: return v ? launch_tile_cfg<Tile3b>(a, st) : launch_tile_cfg<Tile3>(a, st);
-    case 5: return v ? launch_tile_cfg<Tile5b>(a, st) : launch_tile_cfg<Tile5>(a, st);
-    case 7: return v ? launch_tile_cfg<Tile7b>(a, st) : launch_tile_cfg<Tile7>(a, st);
+    case 3: return v == 2 ? launch_tile_cfg<Tile3c>(a, st) : v ? launch_tile_cfg<Tile3b>(a, st) : launch_tile_cfg<Tile3>(a, st);
+    case 5: return v == 2 ? launch_tile_cfg<Tile5c>(a, st) : v ? launch_tile_cfg<Tile5b>(a, st) : launch_tile_cfg<Tile5>(a, st);
+    case 7: return v == 2 ? launch_tile_cfg<Tile7c>(a, st) : v ? launch_tile_cfg<Tile7b>(a, st) : launch_tile_cfg<Tile7>(a, st);
   }
   return cudaErrorNotSupported;
 }

@@ -119,7 +119,7 @@ void layout_padded(const csx_plan_s* p, const int64_t* E, Padded* pd) {
   pd->A[0] = real0 ? (E[0] + 2 * H + 2) : 1;
   pd->A[1] = real1 ? (pd->O[1] + E[1] + 128 + H + 2) : 1;
   const int64_t need2 = pd->O[2] + E[2] + 160 + H + 32;
-  pd->A[2] = 32 * ((need2 + 31) / 32);
+  pd->A[2] = 32 * ((need2 + (p->ndim == 1 ? 2048 : 0) + 31) / 32);  // 1D tiles overhang more
   pd->s1 = pd->A[2];
   pd->s0 = pd->A[1] * pd->A[2];
 }
@@ -256,6 +256,13 @@ csx_status build_pass(const csx_plan_s* p, int tf, Pass* out) {
   // row padded to kc (a multiple of 4) so that every k-slice is 4 consecutive cells of one
   // input row.  Block shape per nk minimises K: nk=3 -> 4x2 (K=24), nk=5 -> 2x4 (K=48),
   // nk=7 -> 4x2 (K=80) versus the paper's 2*ceil(nk^2/4)*4 = 24 / 56 / 104.
+  if (ndim == 1 && P.s2r_ok) {
+    // 1D TC_TILE uses the paper's W_A / W_B fragments unchanged (same GEMM, different M rows)
+    P.tile_ok = 1;
+    P.tile_frags = P.frags;
+    P.tile_ks = P.ks;
+    P.tile_mma_per_pass = P.mma_per_pass;
+  }
   if (ndim >= 2 && nk <= 7) {
     int a = 4, b = 2;
     if (nk == 5) { a = 2; b = 4; }
