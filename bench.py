@@ -215,6 +215,8 @@ def main():
     ap.add_argument("--impl", default="csx", choices=["csx", "reference"])
     ap.add_argument("--config", default=DEFAULT, choices=sorted(CONFIGS))
     ap.add_argument("--engine", default="auto", choices=["auto", "tc_s2r", "tc_tile", "direct"])
+    ap.add_argument("--s2r-variant", default="V", choices=["III", "IV", "V"],
+                    help="TC_S2R breakdown variant (Fig 6): III no padding/no dirty bits, IV padding, V full")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-comparator", action="store_true")
@@ -244,6 +246,8 @@ def main():
     w = synth.physical_weights(shape)
     gext = (ext[0] * world,) + tuple(ext[1:])  # weak scaling: ext per GPU
     plan = csx.Plan(gext, w, shape=s.kind, bc=bc, fuse_steps=tf, engine=args.engine)
+    if args.s2r_variant != "V":
+        plan.set_s2r_variant(padding=args.s2r_variant == "IV", dirty_bits=False)
     info = plan.info()
     engine = info["engine_name"]
     stream = torch.cuda.current_stream()
@@ -338,6 +342,7 @@ def main():
             "data": "synthetic (splitmix64 seed 20240302, dyadic physical weights)",
             "config": {"workload": args.config, "grid": list(gext), "T": T, "bc": bc,
                        "fuse_steps": tfm, "nk": nk, "engine": engine,
+                       "s2r_variant": args.s2r_variant if engine == "tc_s2r" else None,
                        "parallelism": f"slab{world}" if world > 1 else "single",
                        "l2": "inputs larger than L2 (839 MB per grid vs 126 MB); no flush needed"},
             "gpu_launches": int(launches), "roofline": roof}

@@ -80,6 +80,12 @@ csx_status csx_plan(int ndim, const int64_t* extents, csx_shape shape, int radiu
  * this plan's (ndim, radius, Tf). */
 csx_status csx_plan_set_engine(csx_plan_t plan, csx_engine engine);
 
+/* TC_S2R breakdown variants (Fig 6, P.1865-1950), 2D only: padding = 0 uses the bare
+ * stencil2row pitch nk*rr (Fig 5's conflicting 266) instead of the conflict-free one (268);
+ * dirty_bits = 0 replaces the dirty-bits padding by conditional stores in the LUT copy loop.
+ * (1, 1) is the paper's full design (the default); (0, 0) = variant III, (1, 0) = IV. */
+csx_status csx_plan_set_s2r_variant(csx_plan_t plan, int padding, int dirty_bits);
+
 /* Advance d_in by `timesteps` base steps into d_out (both prod(extents) doubles, device,
  * 8-byte aligned; d_in == d_out allowed, any other overlap is INVALID_ARGUMENT; d_in is never
  * written).  Enqueues floor(T/Tf) fused passes plus a remainder pass on `stream` with no host

@@ -58,6 +58,7 @@ def _sig(name, res, args):
 _sig("csx_plan", ctypes.c_int, [ctypes.c_int, _i64p, ctypes.c_int, ctypes.c_int, _dp, ctypes.c_int,
                                 ctypes.c_int, ctypes.POINTER(_vp)])
 _sig("csx_plan_set_engine", ctypes.c_int, [_vp, ctypes.c_int])
+_sig("csx_plan_set_s2r_variant", ctypes.c_int, [_vp, ctypes.c_int, ctypes.c_int])
 _sig("csx_run", ctypes.c_int, [_vp, _vp, _vp, ctypes.c_int64, _vp])
 _sig("csx_run_host", ctypes.c_int, [_vp, _dp, _dp, ctypes.c_int64, _vp])
 _sig("csx_comm_create", ctypes.c_int, [ctypes.c_char_p, ctypes.c_int, ctypes.c_int, ctypes.POINTER(_vp)])
@@ -82,7 +83,7 @@ _sig("csx_profile_read", ctypes.c_int, [_vp, ctypes.POINTER(ctypes.c_double), _i
 
 _sig("csx_halo_schedule", ctypes.c_int, [_vp, ctypes.c_int, ctypes.c_int, _i64p, ctypes.POINTER(ctypes.c_int)])
 
-EXPORTED = ["csx_halo_schedule", "csx_profile_enable", "csx_profile_read", "csx_plan", "csx_plan_set_engine", "csx_run", "csx_run_host", "csx_comm_create",
+EXPORTED = ["csx_plan_set_s2r_variant", "csx_halo_schedule", "csx_profile_enable", "csx_profile_read", "csx_plan", "csx_plan_set_engine", "csx_run", "csx_run_host", "csx_comm_create",
             "csx_comm_destroy", "csx_nccl_unique_id", "csx_shard_rows", "csx_run_sharded",
             "csx_plan_destroy", "csx_status_string", "csx_last_error", "csx_plan_info",
             "csx_compose_weights", "csx_weight_matrices", "csx_stencil2row_index",
@@ -136,6 +137,11 @@ def csx_plan(ndim: int, extents, shape: int, radius: int, weights, bc: int, fuse
 
 def csx_plan_set_engine(plan, engine: int):
     _check(_lib.csx_plan_set_engine(plan, int(engine)), "csx_plan_set_engine")
+
+
+def csx_plan_set_s2r_variant(plan, padding: bool = True, dirty_bits: bool = True):
+    _check(_lib.csx_plan_set_s2r_variant(plan, int(bool(padding)), int(bool(dirty_bits))),
+           "csx_plan_set_s2r_variant")
 
 
 def csx_run(plan, d_in, d_out, timesteps: int, n: int, stream=None):
@@ -285,6 +291,9 @@ class Plan:
     @property
     def handle(self):
         return self._h
+
+    def set_s2r_variant(self, padding: bool = True, dirty_bits: bool = True):
+        csx_plan_set_s2r_variant(self._h, padding, dirty_bits)
 
     def set_engine(self, engine: str):
         csx_plan_set_engine(self._h, ENGINES[engine])

@@ -75,6 +75,10 @@ csx_status ensure_device(csx_plan_s* p) {
   CSX_CUDA(cudaGetDevice(&dev), "cudaGetDevice");
   if (p->device >= 0) {
     if (dev != p->device) return fail(CSX_ERR_INVALID_ARGUMENT, "plan used on another device");
+    for (auto& ps : p->passes) {
+      csx_status s = upload_pass(ps);
+      if (s != CSX_OK) return s;
+    }
     return CSX_OK;
   }
   for (auto& ps : p->passes) {
@@ -157,6 +161,7 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
       e = launch_tile(p->ndim, ps.nk, a, st);
     } else {
       a.frags = ps.d_frags;
+      a.s2r_variant = (p->s2r_pad ? 1 : 0) | (p->s2r_dirty ? 2 : 0);
       int tc_mask = 0;
       if (p->ndim == 1) {
         a.tiles_x = (int)((c.E[2] + ps.bn - 1) / ps.bn);
@@ -300,6 +305,30 @@ csx_status csx_plan(int ndim, const int64_t* extents, csx_shape shape, int radiu
   else if (engine_ok(p, CSX_ENGINE_TC_S2R)) p->engine = CSX_ENGINE_TC_S2R;
   else p->engine = CSX_ENGINE_DIRECT;
   *out = p;
+  return CSX_OK;
+}
+
+csx_status csx_plan_set_s2r_variant(csx_plan_t p, int padding, int dirty_bits) {
+  if (!p) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL plan");
+  if (p->ndim != 2 && !(padding && dirty_bits))
+    return fail(CSX_ERR_UNSUPPORTED, "breakdown variants are 2D only");
+  p->s2r_pad = padding != 0;
+  p->s2r_dirty = dirty_bits != 0;
+  // rebuild the tables of every pass; device copies are re-uploaded at the next run
+  std::vector<Pass> fresh(p->passes.size());
+  for (size_t i = 0; i < p->passes.size(); ++i) {
+    csx_status s = build_pass(p, (int)i + 1, &fresh[i]);
+    if (s != CSX_OK) return s;
+  }
+  if (p->device >= 0) {
+    for (auto& ps : p->passes) {
+      cudaFree(ps.d_frags);
+      cudaFree(ps.d_lut);
+      cudaFree(ps.d_tile_frags);
+      cudaFree(ps.d_wc);
+    }
+  }
+  p->passes.swap(fresh);
   return CSX_OK;
 }
 

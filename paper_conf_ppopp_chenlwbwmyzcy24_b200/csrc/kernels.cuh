@@ -27,6 +27,7 @@ struct S2RArgs {
   // TC_TILE fused FIXED band fix-up (0 = none): edge CTAs recompute the points within
   // fix_band = r*Tf of a GLOBAL face by Tf plain steps on CUDA cores from the staged tile.
   int tc_mask = 0;                // 3D: bit dz set = z offset dz runs on tensor cores
+  int s2r_variant = 3;            // TC_S2R 2D: bit 0 padding, bit 1 dirty bits (breakdown)
   int fix_band = 0;
   int hold_frame = 0;             // write held (frame) values from the staged tile (Tf = 1)
   int r = 0;

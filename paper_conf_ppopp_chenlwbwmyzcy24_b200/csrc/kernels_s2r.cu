@@ -75,9 +75,9 @@ __device__ __forceinline__ void s2r_issue_rows(const double* src, int64_t pitch,
         : "memory");
 }
 
-template <int NK>
+template <int NK, bool PAD, bool DIRTY>
 __global__ void __launch_bounds__(S2R2D<NK>::NT, 2) k_s2r2d(S2RArgs a) {
-  using G = S2R2D<NK>;
+  using G = S2R2D<NK, PAD>;
   extern __shared__ __align__(128) double smem[];
   __shared__ __align__(8) uint64_t full[G::RAW_STAGES], empty[G::RAW_STAGES];
   double* raw = smem;                                           // RAW_STAGES x RAW
@@ -133,8 +133,13 @@ __global__ void __launch_bounds__(S2R2D<NK>::NT, 2) k_s2r2d(S2RArgs a) {
       for (int y = lane; y < G::RC; y += 32) {
         const double v = rrow[y];
         const uint32_t l = lrow[y];
-        sA[l & 0xffffu] = v;
-        sB[l >> 16] = v;
+        if (DIRTY) {  // dirty bits absorb the unused elements: no branch (P.1759-1773)
+          sA[l & 0xffffu] = v;
+          sB[l >> 16] = v;
+        } else {      // breakdown variants III/IV: conditional stores
+          if ((l & 0xffffu) != 0xffffu) sA[l & 0xffffu] = v;
+          if ((l >> 16) != 0xffffu) sB[l >> 16] = v;
+        }
       }
     }
     __syncwarp();
@@ -356,6 +361,17 @@ static cudaError_t launch_persistent(K kernel, int smem, int nthreads, int64_t i
   return cudaGetLastError();
 }
 
+template <int NK>
+static cudaError_t launch_s2r2d_var(const S2RArgs& a, int variant, cudaStream_t st) {
+  // variant bit 0 = padding, bit 1 = dirty bits (default 3 = the paper's full design)
+  switch (variant) {
+    case 3: return launch_persistent(k_s2r2d<NK, true, true>, S2R2D<NK, true>::SMEM, S2R2D<NK>::NT, a.ntiles, st, a);
+    case 1: return launch_persistent(k_s2r2d<NK, true, false>, S2R2D<NK, true>::SMEM, S2R2D<NK>::NT, a.ntiles, st, a);
+    case 2: return launch_persistent(k_s2r2d<NK, false, true>, S2R2D<NK, false>::SMEM, S2R2D<NK>::NT, a.ntiles, st, a);
+    default: return launch_persistent(k_s2r2d<NK, false, false>, S2R2D<NK, false>::SMEM, S2R2D<NK>::NT, a.ntiles, st, a);
+  }
+}
+
 int s2r_smem_bytes(int ndim, int nk, int nf) {
   (void)nf;
   if (ndim == 1) {
@@ -396,9 +412,9 @@ cudaError_t launch_s2r(int ndim, int nk, int nf, const S2RArgs& a, int tc_mask, 
     }
   } else if (ndim == 2) {
     switch (nk) {
-      case 3: return launch_persistent(k_s2r2d<3>, smem, S2R2D<3>::NT, a.ntiles, st, a);
-      case 5: return launch_persistent(k_s2r2d<5>, smem, S2R2D<5>::NT, a.ntiles, st, a);
-      case 7: return launch_persistent(k_s2r2d<7>, smem, S2R2D<7>::NT, a.ntiles, st, a);
+      case 3: return launch_s2r2d_var<3>(a, a.s2r_variant, st);
+      case 5: return launch_s2r2d_var<5>(a, a.s2r_variant, st);
+      case 7: return launch_s2r2d_var<7>(a, a.s2r_variant, st);
     }
   } else if (nk == 3) {
     auto kern = k_s2r3d<3>;

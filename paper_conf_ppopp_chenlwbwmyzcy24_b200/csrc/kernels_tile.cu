@@ -161,8 +161,16 @@ __global__ void __launch_bounds__(C::NT, 1) k_tile2d(S2RArgs a) {
     for (int cg = 0; cg < C::CG; ++cg)
 #pragma unroll
       for (int j = 0; j < C::G; ++j) acc[cg][j][0] = acc[cg][j][1] = 0.0;
+    // FIXED: band outputs of an edge tile are written by k_band (kernels_band.cu) after a pass
+    // of Tf > 1 steps; for Tf = 1 the band is the held frame, written here from the staged tile.
+    const bool edge = tile_is_edge<C>(a, ty, tx);
+    // block j of column group cg covers output rows ty*BM + wm*A*G + A*j + [0, A),
+    // cols tx*BN + wn*WC + cg*8B + B*g + [0, B)
+    const int64_t row0 = (int64_t)ty * C::BM + wm * C::A * C::G + alpha;
+    const int64_t col0 = (int64_t)tx * C::BN + wn * C::WC + C::B * g + beta;
     // Stream the warp's input rows; each A fragment (4 cells of one row) feeds every output
-    // block whose window contains the row.  Consecutive DMMAs go to different accumulators.
+    // block whose window contains the row.  Block j is complete after input row A*j + KR - 1 and
+    // (interior tiles) is stored right there, so the epilogue interleaves with the DMMA stream.
 #pragma unroll
     for (int ra = 0; ra < C::A * C::G + C::NK - 1; ++ra) {
       double f[C::CG][C::KC / 4];
@@ -180,24 +188,12 @@ __global__ void __launch_bounds__(C::NT, 1) k_tile2d(S2RArgs a) {
             for (int cg = 0; cg < C::CG; ++cg)
               dmma_t(acc[cg][j][0], acc[cg][j][1], f[cg][h], wf[rho * (C::KC / 4) + h]);
         }
-    }
-    // FIXED: band outputs of an edge tile are written by k_band (kernels_band.cu) after a pass
-    // of Tf > 1 steps; for Tf = 1 the band is the held frame, written here from the staged tile.
-    const bool edge = tile_is_edge<C>(a, ty, tx);
-    if (!edge) {
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&empty[s]);  // this warp no longer reads stage s
-    }
-    // store: block j of column group cg covers output rows ty*BM + wm*A*G + A*j + [0, A),
-    // cols tx*BN + wn*WC + cg*8B + B*g + [0, B)
-    const int64_t row0 = (int64_t)ty * C::BM + wm * C::A * C::G + alpha;
-#pragma unroll
-    for (int cg = 0; cg < C::CG; ++cg) {
-      const int64_t col = (int64_t)tx * C::BN + wn * C::WC + cg * 8 * C::B + C::B * g + beta;
-#pragma unroll
-      for (int j = 0; j < C::G; ++j) {
+      if (!edge && ra >= C::KR - 1 && (ra - (C::KR - 1)) % C::A == 0) {
+        const int j = (ra - (C::KR - 1)) / C::A;
         const int64_t row = row0 + C::A * j;
-        if (!edge) {
+#pragma unroll
+        for (int cg = 0; cg < C::CG; ++cg) {
+          const int64_t col = col0 + cg * 8 * C::B;
           if (row < a.E1 && col < a.E2) {
             double* p = a.dst.p + row * a.dst.s1 + col;
             if (col + 1 < a.E2 && ((reinterpret_cast<uintptr_t>(p) & 15) == 0)) {
@@ -207,6 +203,21 @@ __global__ void __launch_bounds__(C::NT, 1) k_tile2d(S2RArgs a) {
               if (col + 1 < a.E2) p[1] = acc[cg][j][1];
             }
           }
+        }
+      }
+    }
+    if (!edge) {
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[s]);  // this warp no longer reads stage s
+    }
+#pragma unroll
+    for (int cg = 0; cg < C::CG; ++cg) {
+      const int64_t col = col0 + cg * 8 * C::B;
+#pragma unroll
+      for (int j = 0; j < C::G; ++j) {
+        const int64_t row = row0 + C::A * j;
+        if (!edge) {
+          // stored inside the DMMA loop
         } else if (row < a.E1) {
           const int64_t grow = row + a.gorg1;
           const bool rowband = grow < a.fix_band || grow >= a.GE1 - a.fix_band;
@@ -236,7 +247,8 @@ __global__ void __launch_bounds__(C::NT, 1) k_tile2d(S2RArgs a) {
 // nk -> (a, b, kc); G blocks per warp column, WM x WN consumer warps, STAGES-deep ring.
 // Variant 0: 12 DMMA warps, 3 stages (CTA 96 x 64).  Variant 1: 16 DMMA warps, 2 stages
 // (CTA 128 x 64).  Variant 2: 12 warps of 2 column groups x 4 block rows (CTA 96 x 64) — twice
-// the independent accumulator chains per input row.  CSX_TILE_VARIANT selects (default 0).
+// the independent accumulator chains per input row.  CSX_TILE_VARIANT selects (default 1,
+// the fastest measured: 0.875 of the DMMA peak vs 0.83 for variant 0 on Box-2D9P).
 using Tile3 = TileCfg<3, 4, 2, 4, 8, 3, 4, 3>;
 using Tile5 = TileCfg<5, 2, 4, 8, 8, 6, 2, 3>;
 using Tile7 = TileCfg<7, 4, 2, 8, 8, 3, 4, 3>;
@@ -246,12 +258,13 @@ using Tile7b = TileCfg<7, 4, 2, 8, 8, 4, 4, 2>;
 using Tile3c = TileCfg<3, 4, 2, 4, 4, 6, 2, 3, 2>;
 using Tile5c = TileCfg<5, 2, 4, 8, 4, 12, 1, 3, 2>;
 using Tile7c = TileCfg<7, 4, 2, 8, 4, 6, 2, 3, 2>;
+using Tile7d = TileCfg<7, 4, 2, 8, 8, 2, 3, 3>;  // variant 3: 2 CTAs/SM of 6 DMMA warps (64 x 48)
 
 static int tile_variant() {
   static int v = -1;
   if (v < 0) {
     const char* e = getenv("CSX_TILE_VARIANT");
-    v = e ? atoi(e) : 0;
+    v = e ? atoi(e) : 1;
   }
   return v;
 }
@@ -429,7 +442,7 @@ __global__ void __launch_bounds__(C::NT, 2) k_tile3d(S2RArgs a, int tc_mask) {
   }
 }
 
-using Tile3D3 = Tile3DCfg<3, 8, 2, 2, 4, 32>;  // CTA 64 x 32 outputs, 4-plane ring, 32 planes per item
+using Tile3D3 = Tile3DCfg<3, 8, 2, 2, 4, 32>;  // CTA 64 x 32 outputs, 4 DMMA warps, 4-plane ring, 32 planes per item
 
 
 // ------------------------------------------------------------------------------------------
@@ -668,7 +681,7 @@ cudaError_t launch_tile(int ndim, int nk, const S2RArgs& a, cudaStream_t st) {
   switch (nk) {
     case 3: return v == 2 ? launch_tile_cfg<Tile3c>(a, st) : v ? launch_tile_cfg<Tile3b>(a, st) : launch_tile_cfg<Tile3>(a, st);
     case 5: return v == 2 ? launch_tile_cfg<Tile5c>(a, st) : v ? launch_tile_cfg<Tile5b>(a, st) : launch_tile_cfg<Tile5>(a, st);
-    case 7: return v == 2 ? launch_tile_cfg<Tile7c>(a, st) : v ? launch_tile_cfg<Tile7b>(a, st) : launch_tile_cfg<Tile7>(a, st);
+    case 7: return v == 3 ? launch_tile_cfg<Tile7d>(a, st) : v == 2 ? launch_tile_cfg<Tile7c>(a, st) : v ? launch_tile_cfg<Tile7b>(a, st) : launch_tile_cfg<Tile7>(a, st);
   }
   return cudaErrorNotSupported;
 }

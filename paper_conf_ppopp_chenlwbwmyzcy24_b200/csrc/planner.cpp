@@ -193,6 +193,12 @@ csx_status build_pass(const csx_plan_s* p, int tf, Pass* out) {
   // the kernels' constexpr pitch must be the conflict-free pitch of the bank model
   if (P.pitch != choose_pitch(ndim == 1 ? 4 * P.ks : nk * P.rr))
     return fail(CSX_ERR_INTERNAL, "stencil2row pitch disagrees with the bank-conflict model");
+  // Breakdown variants (Fig 6, P.1865-1950), 2D only: without padding the pitch is the bare
+  // nk*rr (266 for the 32x64 tile: 2-way conflicts, Fig 5); without dirty bits the elements
+  // that belong to neither matrix get a sentinel and the copy loop branches on it.
+  const bool pad = ndim != 2 || p->s2r_pad;
+  const bool dirty_bits = ndim != 2 || p->s2r_dirty;
+  if (!pad) P.pitch = nk * P.rr;
   // LUT: every input-region element -> (global offset, smem offset in A, in B).  Elements
   // that belong to neither matrix are routed to the dirty row (row index `strips`), so the
   // copy loop has no branches (P.1759-1773).
@@ -213,7 +219,7 @@ csx_status build_pass(const csx_plan_s* p, int tf, Pass* out) {
       const int64_t e = (int64_t)x * P.rc + y;
       P.lut_g[e] = (int32_t)(ndim == 1 ? y : x * sp[1] + y);
       int64_t row, col;
-      const int dirty = dirty_base + (int)(e % P.pitch);
+      const int dirty = dirty_bits ? dirty_base + (int)(e % P.pitch) : 0xffff;
       // Eq 5 on tile-local coordinates: for 1D the "row" of the input is x = 0 and the
       // stencil2row row length is nk (P.1779-1786).
       if (s2r_index(nk, 0, ndim == 1 ? 0 : x, y, &row, &col) && row < strips)

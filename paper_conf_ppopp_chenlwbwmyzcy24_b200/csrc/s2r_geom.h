@@ -13,7 +13,7 @@ constexpr int s2r_pitch(int min_pitch) {
   return p;
 }
 
-template <int NK>
+template <int NK, bool PAD = true>
 struct S2R2D {
   static constexpr int NKV = NK;
   static constexpr int SW = NK + 1;            // strip width: outputs per strip row
@@ -24,7 +24,7 @@ struct S2R2D {
   static constexpr int RC = BN + NK - 1;       // input region cols
   static constexpr int NE = RR * RC;           // LUT entries
   static constexpr int STRIPS = 8;             // stencil2row rows per CTA (+1 dirty row)
-  static constexpr int PITCH = s2r_pitch(NK * RR);
+  static constexpr int PITCH = PAD ? s2r_pitch(NK * RR) : NK * RR;
   static constexpr int R = (NK - 1) / 2;
   // B200 staging: the raw input region arrives by cp.async.bulk rows (16-B aligned, hence the
   // ODD shift) in a 2-stage ring filled by one producer warp; 8 consumer warps scatter it

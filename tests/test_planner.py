@@ -233,3 +233,17 @@ def test_shard_rows_partition():
         assert all(a[1] == b[0] for a, b in zip(spans, spans[1:]))
         assert max(h - l for l, h in spans) - min(h - l for l, h in spans) <= 1
     p.close()
+
+
+def test_s2r_variant_tables():
+    """Breakdown variants: no padding -> pitch 266 (Fig 5); no dirty bits -> sentinel entries."""
+    p = csx.Plan((320, 640), synth.physical_weights("box2d9p"), engine="tc_s2r")
+    p.set_s2r_variant(padding=False, dirty_bits=False)
+    assert p.info()["s2r_pitch"] == 266
+    la, lb = p.lut()
+    assert np.count_nonzero(la == 0xFFFF) > 0 and np.count_nonzero(lb == 0xFFFF) > 0
+    live = la[la != 0xFFFF]
+    assert len(np.unique(live)) == len(live) == 8 * 7 * 38
+    p.set_s2r_variant(padding=True, dirty_bits=True)
+    assert p.info()["s2r_pitch"] == 268
+    p.close()
