@@ -128,6 +128,8 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
       CSX_CUDA(cudaEventRecord(ev0, st), "cudaEventRecord");
     }
     S2RArgs a;
+    a.part = eng == CSX_ENGINE_TC_TILE ? c.part : 0;
+    a.max_ctas = c.max_ctas;
     a.src = c.src;
     a.dst = c.dst;
     a.E0 = c.E[0]; a.E1 = c.E[1]; a.E2 = c.E[2];
@@ -186,6 +188,7 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
   }
   const bool direct_all = eng == CSX_ENGINE_DIRECT;
   const int real[3] = {p->ndim == 3, p->ndim >= 2, 1};
+  if (eng == CSX_ENGINE_TC_TILE && c.part == 1) return CSX_OK;  // fix-ups run with the edge part
   if (direct_all) {
     DirectArgs d;
     d.src = c.src;

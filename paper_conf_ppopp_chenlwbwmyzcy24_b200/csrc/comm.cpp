@@ -11,6 +11,7 @@
 #include <cuda_runtime.h>
 #include <nccl.h>
 
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <vector>
@@ -22,6 +23,9 @@
 struct csx_comm_s {
   ncclComm_t comm = nullptr;
   int rank = 0, nranks = 1;
+  cudaStream_t cs = nullptr;       // halo-exchange stream (overlaps the interior kernels)
+  cudaEvent_t ev_edge = nullptr;   // compute -> comm: this pass's edge tiles are written
+  cudaEvent_t ev_x = nullptr;      // comm -> compute: the next pass's ghosts have arrived
 };
 
 namespace csx {
@@ -113,6 +117,13 @@ csx_status csx_comm_create(const void* nccl_unique_id, int rank, int nranks, csx
   }
   c->rank = rank;
   c->nranks = nranks;
+  if (cudaStreamCreateWithFlags(&c->cs, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_edge, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_x, cudaEventDisableTiming) != cudaSuccess) {
+    ncclCommDestroy(c->comm);
+    delete c;
+    return fail(CSX_ERR_CUDA, "comm stream / event creation failed");
+  }
   *out = c;
   return CSX_OK;
 }
@@ -120,6 +131,9 @@ csx_status csx_comm_create(const void* nccl_unique_id, int rank, int nranks, csx
 csx_status csx_comm_destroy(csx_comm_t c) {
   if (!c) return CSX_OK;
   if (c->comm) ncclCommDestroy(c->comm);
+  if (c->ev_edge) cudaEventDestroy(c->ev_edge);
+  if (c->ev_x) cudaEventDestroy(c->ev_x);
+  if (c->cs) cudaStreamDestroy(c->cs);
   delete c;
   return CSX_OK;
 }
@@ -209,6 +223,14 @@ csx_status csx_run_sharded(csx_plan_t p, csx_comm_t c, const double* d_in, doubl
   const int rem = (int)(T % p->tf);
   const int64_t npass = nmain + (rem ? 1 : 0);
   const View out{d_out, El[1] * El[2], El[2]};
+  // TC_TILE overlaps the halo exchange of pass i+1 with the interior tiles of pass i+1:
+  //   compute: interior(i) -> [wait ghosts(i)] -> edge(i) + fix-ups -> ghost fill -> ev_edge
+  //   comm:    [wait ev_edge] -> exchange into dst(i) -> ev_x
+  // interior tiles never read ghost rows; edge tiles are the first / last slab tiles.
+  // (CSX_FORCE_OVERLAP=1 exercises the overlapped schedule on a single rank, for tests)
+  const char* fo = getenv("CSX_FORCE_OVERLAP");
+  const bool overlap = p->engine == CSX_ENGINE_TC_TILE && (c->nranks > 1 || (fo && fo[0] == '1'));
+  const int max_ctas = overlap ? num_sms() - 2 : 0;  // leave SMs for the NCCL kernels
   int cur = 0;
   for (int64_t i = 0; i < npass; ++i) {
     const int tfp = i < nmain ? p->tf : rem;
@@ -218,11 +240,39 @@ csx_status csx_run_sharded(csx_plan_t p, csx_comm_t c, const double* d_in, doubl
     pc.dst = last ? out : b[cur ^ 1];
     for (int a = 0; a < 3; ++a) { pc.E[a] = El[a]; pc.gorg[a] = 0; }
     pc.gorg[a0] = lo;
-    s = run_pass(p, p->passes[tfp - 1], pc, st);
-    if (s != CSX_OK) return s;
-    if (!last) {
-      s = refresh(cur ^ 1);
+    if (!overlap) {
+      s = run_pass(p, p->passes[tfp - 1], pc, st);
       if (s != CSX_OK) return s;
+      if (!last) {
+        s = refresh(cur ^ 1);
+        if (s != CSX_OK) return s;
+      }
+    } else {
+      pc.max_ctas = max_ctas;
+      pc.part = 1;
+      s = run_pass(p, p->passes[tfp - 1], pc, st);
+      if (s != CSX_OK) return s;
+      if (i > 0) {
+        cudaError_t e2 = cudaStreamWaitEvent(st, c->ev_x, 0);
+        if (e2 != cudaSuccess) return cuda_fail(e2, "wait halo");
+      }
+      pc.part = 2;
+      s = run_pass(p, p->passes[tfp - 1], pc, st);
+      if (s != CSX_OK) return s;
+      if (!last) {
+        if (p->bc == CSX_BC_PERIODIC) {
+          cudaError_t e2 = launch_ghost_fill(b[cur ^ 1], El, real, fill, p->halo, st);
+          if (e2 != cudaSuccess) return cuda_fail(e2, "ghost fill");
+          p->n_launches += (real[0] && fill[0]) + (real[1] && fill[1]) + fill[2];
+        }
+        cudaError_t e2 = cudaEventRecord(c->ev_edge, st);
+        if (e2 == cudaSuccess) e2 = cudaStreamWaitEvent(c->cs, c->ev_edge, 0);
+        if (e2 != cudaSuccess) return cuda_fail(e2, "edge event");
+        s = exchange(p, c, p->d_sbuf[cur ^ 1], a0, El[a0], c->cs);
+        if (s != CSX_OK) return s;
+        e2 = cudaEventRecord(c->ev_x, c->cs);
+        if (e2 != cudaSuccess) return cuda_fail(e2, "halo event");
+      }
     }
     cur ^= 1;
   }

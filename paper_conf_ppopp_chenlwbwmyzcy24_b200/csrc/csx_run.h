@@ -15,6 +15,8 @@ struct PassCtx {
   View dst;                       // destination at its interior origin
   int64_t E[3];                   // local interior extents (normalised)
   int64_t gorg[3];                // local origin in global coordinates (slab offset)
+  int part = 0;                   // TC_TILE slab-tile subset: 0 all, 1 interior, 2 edge (+ fix-ups)
+  int max_ctas = 0;               // persistent-grid cap (leaves SMs to NCCL while overlapping)
 };
 
 csx_status cuda_fail(cudaError_t e, const char* where);

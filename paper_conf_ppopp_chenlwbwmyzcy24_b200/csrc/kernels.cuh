@@ -27,6 +27,11 @@ struct S2RArgs {
   // TC_TILE fused FIXED band fix-up (0 = none): edge CTAs recompute the points within
   // fix_band = r*Tf of a GLOBAL face by Tf plain steps on CUDA cores from the staged tile.
   int tc_mask = 0;                // 3D: bit dz set = z offset dz runs on tensor cores
+  // slab-axis tile subset (sharded overlap): part 0 = all, 1 = interior (no ghost reads),
+  // 2 = edge (the first / last slab tiles, whose halo reaches the exchanged ghost rows)
+  int part = 0;
+  int max_ctas = 0;               // cap on the persistent grid (0 = all SMs)
+  int64_t ra0 = 0, ra1 = 0, rb0 = 0, rb1 = 0;  // slab-tile ranges, filled by the launcher
   int s2r_variant = 3;            // TC_S2R 2D: bit 0 padding, bit 1 dirty bits (breakdown)
   int fix_band = 0;
   int hold_frame = 0;             // write held (frame) values from the staged tile (Tf = 1)

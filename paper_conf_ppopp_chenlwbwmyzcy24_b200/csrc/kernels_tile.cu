@@ -67,6 +67,40 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(bar)) : "memory");
 }
 
+// slab tile k of this launch -> slab tile index (ranges A then B, see S2RArgs::part)
+__device__ __forceinline__ int64_t slab_map(const S2RArgs& a, int64_t k) {
+  const int64_t na = a.ra1 - a.ra0;
+  return k < na ? a.ra0 + k : a.rb0 + (k - na);
+}
+
+// host: fill the slab-tile ranges for part (0 all, 1 interior, 2 edge); n slab tiles of `size`
+// outputs along the slab axis of local length El, halo R.  Returns the number of slab tiles.
+static int64_t set_ranges(S2RArgs& a, int64_t n, int64_t size, int64_t El, int R) {
+  int64_t e1 = n;  // first tile of the trailing edge run
+  while (e1 > 0 && e1 * size + R > El) --e1;
+  // tile k is "edge" if k == 0 or k >= e1 (k*size - R < 0 or (k+1)*size + R > El)
+  a.ra0 = a.ra1 = a.rb0 = a.rb1 = 0;
+  if (a.part == 0 || e1 <= 1) {
+    if (a.part == 1) return 0;  // no interior
+    a.ra0 = 0;
+    a.ra1 = n;
+  } else if (a.part == 1) {
+    a.ra0 = 1;
+    a.ra1 = e1;
+  } else {
+    a.ra0 = 0;
+    a.ra1 = 1;
+    a.rb0 = e1;
+    a.rb1 = n;
+  }
+  return (a.ra1 - a.ra0) + (a.rb1 - a.rb0);
+}
+
+static int64_t cap_grid(const S2RArgs& a, int64_t grid) {
+  if (a.max_ctas > 0 && grid > a.max_ctas) grid = a.max_ctas;
+  return grid;
+}
+
 constexpr int s2r_pitch_dev(int min_pitch) {
   int p = min_pitch;
   while (p % 16 != 4 && p % 16 != 12) ++p;
@@ -97,8 +131,9 @@ struct TileCfg {
 template <class C>
 __device__ __forceinline__ void issue_tile(const S2RArgs& a, int64_t tile, double* stage,
                                            uint64_t* bar, int lane) {
-  const int ty = (int)(tile / a.tiles_x);
-  const int tx = (int)(tile - (int64_t)ty * a.tiles_x);
+  const int64_t tyl = tile / a.tiles_x;
+  const int tx = (int)(tile - tyl * a.tiles_x);
+  const int ty = (int)slab_map(a, tyl);
   const double* src = a.src.p + (int64_t)(ty * C::BM - C::R) * a.src.s1 + (tx * C::BN - C::R - C::ODD);
   if (lane == 0) mbar_expect_tx(bar, (uint32_t)(C::STAGE * 8));
   __syncwarp();
@@ -152,8 +187,9 @@ __global__ void __launch_bounds__(C::NT, 1) k_tile2d(S2RArgs a) {
   for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
     const int s = it % C::STAGES;
     mbar_wait(&full[s], (it / C::STAGES) & 1);
-    const int ty = (int)(tile / a.tiles_x);
-    const int tx = (int)(tile - (int64_t)ty * a.tiles_x);
+    const int64_t tyl = tile / a.tiles_x;
+    const int tx = (int)(tile - tyl * a.tiles_x);
+    const int ty = (int)slab_map(a, tyl);
     const double* base = smem + s * C::STAGE + (wm * C::A * C::G) * C::TP + wn * C::WC + C::ODD +
                          C::B * g + t;
     double acc[C::CG][C::G][2];
@@ -322,7 +358,8 @@ __global__ void __launch_bounds__(C::NT, 2) k_tile3d(S2RArgs a, int tc_mask) {
   if (warp == C::NCW) {  // producer: planes of every work item, in consumption order
     int64_t q = 0;
     for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
-      const int64_t zc = item / ncol, tile = item - zc * ncol;
+      const int64_t zcl = item / ncol, tile = item - zcl * ncol;
+      const int64_t zc = slab_map(a, zcl);
       const int ty = (int)(tile / a.tiles_x), tx = (int)(tile - (int64_t)ty * a.tiles_x);
       const int64_t z0 = zc * C::ZCH, z1 = min(a.E0, z0 + C::ZCH);
       for (int64_t zi = z0 - C::R; zi < z1 + C::R; ++zi, ++q) {
@@ -348,7 +385,8 @@ __global__ void __launch_bounds__(C::NT, 2) k_tile3d(S2RArgs a, int tc_mask) {
   const bool any_cuda = tc_mask != (1 << C::NK) - 1;
   int64_t q0 = 0;  // plane sequence number of the current item's first plane
   for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
-    const int64_t zc = item / ncol, tile = item - zc * ncol;
+    const int64_t zcl = item / ncol, tile = item - zcl * ncol;
+    const int64_t zc = slab_map(a, zcl);
     const int ty = (int)(tile / a.tiles_x), tx = (int)(tile - (int64_t)ty * a.tiles_x);
     const int64_t z0 = zc * C::ZCH, z1 = min(a.E0, z0 + C::ZCH);
     const int64_t col = (int64_t)tx * C::BN + wn * 8 * C::B + C::B * g + beta;
@@ -488,7 +526,7 @@ __global__ void __launch_bounds__(C::NT, 2) k_tile1d(S2RArgs a) {
     for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
       const int s = it % C::STAGES, n = it / C::STAGES;
       if (n > 0) mbar_wait(&empty[s], (n - 1) & 1);
-      const int64_t t0 = tile * C::TILE;
+      const int64_t t0 = slab_map(a, tile) * C::TILE;
       int nseg = (int)min((int64_t)8, (a.E2 - t0 + C::L - 1) / C::L);
       if (lane == 0) mbar_expect_tx(&full[s], (uint32_t)(nseg * C::SL * 8));
       __syncwarp();
@@ -513,7 +551,8 @@ __global__ void __launch_bounds__(C::NT, 2) k_tile1d(S2RArgs a) {
     const int s = it % C::STAGES;
     mbar_wait(&full[s], (it / C::STAGES) & 1);
     const double* seg = smem + s * C::STAGE + g * C::P + C::ODD + t;  // this lane's segment g
-    const int64_t t0 = tile * C::TILE + (int64_t)g * C::L;
+    const int64_t tsl = slab_map(a, tile);
+    const int64_t t0 = tsl * C::TILE + (int64_t)g * C::L;
     constexpr int NSTRIP = C::L / C::SW;
     double res[(NSTRIP + C::NCW - 1) / C::NCW][C::NF][2];
 #pragma unroll
@@ -537,7 +576,7 @@ __global__ void __launch_bounds__(C::NT, 2) k_tile1d(S2RArgs a) {
     // FIXED: the band b = r*Tf at each global end is recomputed by Tf plain steps (reading A1)
     // by warp 0 from the staged segments, one lane per point, neighbours via shuffles.
     const int fb = a.fix_band;
-    const int64_t tg0 = tile * C::TILE + a.gorg2;  // global index of the tile's first output
+    const int64_t tg0 = tsl * C::TILE + a.gorg2;  // global index of the tile's first output
     if (fb > 0 && warp == 0 && (tg0 < fb || tg0 + C::TILE > a.GE2 - fb)) {
       const int r = a.r, tf = fb / r, D = r * (tf - 1);
       for (int sg = 0; sg < 8; ++sg) {
@@ -608,13 +647,14 @@ __global__ void __launch_bounds__(C::NT, 2) k_tile1d(S2RArgs a) {
 
 template <class C>
 static cudaError_t launch_tile1d_cfg(S2RArgs a, cudaStream_t st) {
-  a.ntiles = (a.E2 + C::TILE - 1) / C::TILE;
+  a.ntiles = set_ranges(a, (a.E2 + C::TILE - 1) / C::TILE, C::TILE, a.E2, C::R);
+  if (a.ntiles == 0) return cudaSuccess;
   cudaError_t e = cudaFuncSetAttribute(k_tile1d<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
   if (e != cudaSuccess) return e;
   int occ = 0;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_tile1d<C>, C::NT, C::SMEM);
   if (e != cudaSuccess) return e;
-  int64_t grid = (int64_t)(occ < 1 ? 1 : occ) * num_sms();
+  int64_t grid = cap_grid(a, (int64_t)(occ < 1 ? 1 : occ) * num_sms());
   if (grid > a.ntiles) grid = a.ntiles;
   k_tile1d<C><<<(unsigned)grid, C::NT, C::SMEM, st>>>(a);
   return cudaGetLastError();
@@ -642,13 +682,14 @@ template <class C>
 static cudaError_t launch_tile_cfg(S2RArgs a, cudaStream_t st) {
   a.tiles_x = (int)((a.E2 + C::BN - 1) / C::BN);
   a.tiles_y = (int)((a.E1 + C::BM - 1) / C::BM);
-  a.ntiles = (int64_t)a.tiles_x * a.tiles_y;
+  a.ntiles = (int64_t)a.tiles_x * set_ranges(a, a.tiles_y, C::BM, a.E1, C::R);
+  if (a.ntiles == 0) return cudaSuccess;
   cudaError_t e = cudaFuncSetAttribute(k_tile2d<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
   if (e != cudaSuccess) return e;
   int occ = 0;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_tile2d<C>, C::NT, C::SMEM);
   if (e != cudaSuccess) return e;
-  int64_t grid = (int64_t)(occ < 1 ? 1 : occ) * num_sms();
+  int64_t grid = cap_grid(a, (int64_t)(occ < 1 ? 1 : occ) * num_sms());
   if (grid > a.ntiles) grid = a.ntiles;
   k_tile2d<C><<<(unsigned)grid, C::NT, C::SMEM, st>>>(a);
   return cudaGetLastError();
@@ -658,13 +699,14 @@ template <class C>
 static cudaError_t launch_tile3d_cfg(S2RArgs a, int tc_mask, cudaStream_t st) {
   a.tiles_x = (int)((a.E2 + C::BN - 1) / C::BN);
   a.tiles_y = (int)((a.E1 + C::BM - 1) / C::BM);
-  a.ntiles = (int64_t)a.tiles_x * a.tiles_y * ((a.E0 + C::ZCH - 1) / C::ZCH);
+  a.ntiles = (int64_t)a.tiles_x * a.tiles_y * set_ranges(a, (a.E0 + C::ZCH - 1) / C::ZCH, C::ZCH, a.E0, C::R);
+  if (a.ntiles == 0) return cudaSuccess;
   cudaError_t e = cudaFuncSetAttribute(k_tile3d<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
   if (e != cudaSuccess) return e;
   int occ = 0;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_tile3d<C>, C::NT, C::SMEM);
   if (e != cudaSuccess) return e;
-  int64_t grid = (int64_t)(occ < 1 ? 1 : occ) * num_sms();
+  int64_t grid = cap_grid(a, (int64_t)(occ < 1 ? 1 : occ) * num_sms());
   if (grid > a.ntiles) grid = a.ntiles;
   k_tile3d<C><<<(unsigned)grid, C::NT, C::SMEM, st>>>(a, tc_mask);
   return cudaGetLastError();

@@ -217,3 +217,25 @@ def test_s2r_breakdown_variants(csx, pad, dirty):
         torch.cuda.synchronize()
         p.close()
         assert rel(d_out.cpu().numpy(), oracle.run(u0, w, "fixed", 7)) <= TOL, (name, pad, dirty)
+
+
+@pytest.mark.parametrize("name,ext,T", [("box2d9p", (400, 130), 10), ("heat1d", (30000,), 23),
+                                        ("box3d27p", (100, 30, 40), 4), ("box2d49p", (300, 90), 3)])
+@pytest.mark.parametrize("bc", ["fixed", "periodic"])
+def test_sharded_overlap_schedule(csx, monkeypatch, name, ext, T, bc):
+    """The overlapped sharded schedule (interior tiles, then edge tiles after the halo event,
+    exchange on its own stream) forced on one rank: same result as the oracle."""
+    monkeypatch.setenv("CSX_FORCE_OVERLAP", "1")
+    s = synth.SHAPES[name]
+    w = synth.random_weights(name)
+    u0 = synth.grid(ext, seed=14)
+    p = csx.Plan(u0.shape, w, shape=s.kind, bc=bc)
+    assert p.info()["engine_name"] == "tc_tile"
+    comm = csx.csx_comm_create(csx.csx_nccl_unique_id(), 0, 1)
+    d_in = torch.from_numpy(u0).cuda()
+    d_out = torch.empty_like(d_in)
+    p.run_sharded(comm, d_in, d_out, T, u0.size)
+    torch.cuda.synchronize()
+    csx.csx_comm_destroy(comm)
+    p.close()
+    assert rel(d_out.cpu().numpy(), oracle.run(u0, w, bc, T)) <= TOL, (name, bc)
