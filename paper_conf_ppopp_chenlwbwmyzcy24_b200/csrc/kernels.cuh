@@ -31,6 +31,7 @@ struct S2RArgs {
   // 2 = edge (the first / last slab tiles, whose halo reaches the exchanged ghost rows)
   int part = 0;
   int max_ctas = 0;               // cap on the persistent grid (0 = all SMs)
+  int dst_aligned = 0;            // dst rows are 16-B aligned (unguarded double2 stores)
   int64_t ra0 = 0, ra1 = 0, rb0 = 0, rb1 = 0;  // slab-tile ranges, filled by the launcher
   int s2r_variant = 3;            // TC_S2R 2D: bit 0 padding, bit 1 dirty bits (breakdown)
   int fix_band = 0;

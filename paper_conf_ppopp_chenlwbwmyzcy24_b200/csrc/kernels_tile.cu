@@ -204,6 +204,8 @@ __global__ void __launch_bounds__(C::NT, 1) k_tile2d(S2RArgs a) {
     // cols tx*BN + wn*WC + cg*8B + B*g + [0, B)
     const int64_t row0 = (int64_t)ty * C::BM + wm * C::A * C::G + alpha;
     const int64_t col0 = (int64_t)tx * C::BN + wn * C::WC + C::B * g + beta;
+    const bool full_tile = a.dst_aligned && (int64_t)(ty + 1) * C::BM <= a.E1 &&
+                           (int64_t)(tx + 1) * C::BN <= a.E2;
     // Stream the warp's input rows; each A fragment (4 cells of one row) feeds every output
     // block whose window contains the row.  Block j is complete after input row A*j + KR - 1 and
     // (interior tiles) is stored right there, so the epilogue interleaves with the DMMA stream.
@@ -230,7 +232,10 @@ __global__ void __launch_bounds__(C::NT, 1) k_tile2d(S2RArgs a) {
 #pragma unroll
         for (int cg = 0; cg < C::CG; ++cg) {
           const int64_t col = col0 + cg * 8 * C::B;
-          if (row < a.E1 && col < a.E2) {
+          if (full_tile) {  // whole tile inside the grid, 16-B aligned rows: unguarded stores
+            *reinterpret_cast<double2*>(a.dst.p + row * a.dst.s1 + col) =
+                make_double2(acc[cg][j][0], acc[cg][j][1]);
+          } else if (row < a.E1 && col < a.E2) {
             double* p = a.dst.p + row * a.dst.s1 + col;
             if (col + 1 < a.E2 && ((reinterpret_cast<uintptr_t>(p) & 15) == 0)) {
               *reinterpret_cast<double2*>(p) = make_double2(acc[cg][j][0], acc[cg][j][1]);
@@ -680,6 +685,7 @@ bool tile_kernel_exists(int ndim, int nk) {
 
 template <class C>
 static cudaError_t launch_tile_cfg(S2RArgs a, cudaStream_t st) {
+  a.dst_aligned = ((reinterpret_cast<uintptr_t>(a.dst.p) & 15) == 0) && (a.dst.s1 % 2 == 0);
   a.tiles_x = (int)((a.E2 + C::BN - 1) / C::BN);
   a.tiles_y = (int)((a.E1 + C::BM - 1) / C::BM);
   a.ntiles = (int64_t)a.tiles_x * set_ranges(a, a.tiles_y, C::BM, a.E1, C::R);
