@@ -108,9 +108,11 @@ constexpr int s2r_pitch_dev(int min_pitch) {
 }
 
 // Compile-time geometry of one TC_TILE instantiation.
-template <int NK_, int A_, int B_, int KC_, int G_, int WM_, int WN_, int STAGES_, int CG_ = 1>
+template <int NK_, int A_, int B_, int KC_, int G_, int WM_, int WN_, int STAGES_, int CG_ = 1,
+          int MINB_ = 1>
 struct TileCfg {
   static constexpr int NK = NK_, A = A_, B = B_, KC = KC_, G = G_, WM = WM_, WN = WN_;
+  static constexpr int MINB = MINB_;                // CTAs per SM the registers are sized for
   static constexpr int STAGES = STAGES_;
   static constexpr int CG = CG_;                    // 8-block column groups per warp
   static constexpr int R = (NK - 1) / 2;
@@ -152,7 +154,7 @@ __device__ __forceinline__ bool tile_is_edge(const S2RArgs& a, int ty, int tx) {
 // Warp-specialised persistent kernel: warp NCW is the producer (bulk copies of the input tile
 // into a STAGES-deep smem ring, full/empty mbarriers); warps 0..NCW-1 run the DMMA GEMM.
 template <class C>
-__global__ void __launch_bounds__(C::NT, 1) k_tile2d(S2RArgs a) {
+__global__ void __launch_bounds__(C::NT, C::MINB) k_tile2d(S2RArgs a) {
   extern __shared__ __align__(128) double smem[];
   __shared__ __align__(8) uint64_t full[C::STAGES], empty[C::STAGES];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -299,7 +301,8 @@ using Tile7b = TileCfg<7, 4, 2, 8, 8, 4, 4, 2>;
 using Tile3c = TileCfg<3, 4, 2, 4, 4, 6, 2, 3, 2>;
 using Tile5c = TileCfg<5, 2, 4, 8, 4, 12, 1, 3, 2>;
 using Tile7c = TileCfg<7, 4, 2, 8, 4, 6, 2, 3, 2>;
-using Tile7d = TileCfg<7, 4, 2, 8, 8, 2, 3, 3>;  // variant 3: 2 CTAs/SM of 6 DMMA warps (64 x 48)
+using Tile7d = TileCfg<7, 4, 2, 8, 8, 2, 3, 3, 1, 2>;  // variant 3: 2 CTAs/SM of 6 DMMA warps (64 x 48)
+using Tile7e = TileCfg<7, 4, 2, 8, 8, 2, 4, 2, 1, 2>;  // variant 4: 2 CTAs/SM of 8 DMMA warps (64 x 64)
 
 static int tile_variant() {
   static int v = -1;
@@ -485,7 +488,7 @@ __global__ void __launch_bounds__(C::NT, 2) k_tile3d(S2RArgs a, int tc_mask) {
   }
 }
 
-using Tile3D3 = Tile3DCfg<3, 8, 2, 2, 4, 32>;  // CTA 64 x 32 outputs, 4 DMMA warps, 4-plane ring, 32 planes per item
+using Tile3D3 = Tile3DCfg<3, 8, 2, 2, 5, 32>;  // CTA 64 x 32 outputs, 4 DMMA warps, 4-plane ring, 32 planes per item
 
 
 // ------------------------------------------------------------------------------------------
@@ -514,7 +517,7 @@ struct Tile1DCfg {
 };
 
 template <class C>
-__global__ void __launch_bounds__(C::NT, 2) k_tile1d(S2RArgs a) {
+__global__ void __launch_bounds__(C::NT, 2) k_tile1d(S2RArgs a) {  // 2 CTAs/SM
   extern __shared__ __align__(128) double smem[];
   __shared__ __align__(8) uint64_t full[C::STAGES], empty[C::STAGES];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -667,13 +670,13 @@ static cudaError_t launch_tile1d_cfg(S2RArgs a, cudaStream_t st) {
 
 static cudaError_t launch_tile1d(int nk, const S2RArgs& a, cudaStream_t st) {
   switch (nk) {
-    case 3: return launch_tile1d_cfg<Tile1DCfg<3, 256, 4, 6>>(a, st);
-    case 5: return launch_tile1d_cfg<Tile1DCfg<5, 252, 4, 6>>(a, st);
-    case 7: return launch_tile1d_cfg<Tile1DCfg<7, 256, 4, 6>>(a, st);
-    case 9: return launch_tile1d_cfg<Tile1DCfg<9, 250, 4, 6>>(a, st);
-    case 11: return launch_tile1d_cfg<Tile1DCfg<11, 252, 4, 6>>(a, st);
-    case 13: return launch_tile1d_cfg<Tile1DCfg<13, 252, 4, 6>>(a, st);
-    case 15: return launch_tile1d_cfg<Tile1DCfg<15, 256, 4, 6>>(a, st);
+    case 3: return launch_tile1d_cfg<Tile1DCfg<3, 256, 8, 5>>(a, st);
+    case 5: return launch_tile1d_cfg<Tile1DCfg<5, 252, 8, 5>>(a, st);
+    case 7: return launch_tile1d_cfg<Tile1DCfg<7, 256, 8, 5>>(a, st);
+    case 9: return launch_tile1d_cfg<Tile1DCfg<9, 250, 8, 5>>(a, st);
+    case 11: return launch_tile1d_cfg<Tile1DCfg<11, 252, 8, 5>>(a, st);
+    case 13: return launch_tile1d_cfg<Tile1DCfg<13, 252, 8, 5>>(a, st);
+    case 15: return launch_tile1d_cfg<Tile1DCfg<15, 256, 8, 5>>(a, st);
   }
   return cudaErrorNotSupported;
 }
@@ -729,7 +732,7 @@ cudaError_t launch_tile(int ndim, int nk, const S2RArgs& a, cudaStream_t st) {
   switch (nk) {
     case 3: return v == 2 ? launch_tile_cfg<Tile3c>(a, st) : v ? launch_tile_cfg<Tile3b>(a, st) : launch_tile_cfg<Tile3>(a, st);
     case 5: return v == 2 ? launch_tile_cfg<Tile5c>(a, st) : v ? launch_tile_cfg<Tile5b>(a, st) : launch_tile_cfg<Tile5>(a, st);
-    case 7: return v == 3 ? launch_tile_cfg<Tile7d>(a, st) : v == 2 ? launch_tile_cfg<Tile7c>(a, st) : v ? launch_tile_cfg<Tile7b>(a, st) : launch_tile_cfg<Tile7>(a, st);
+    case 7: return v == 4 ? launch_tile_cfg<Tile7e>(a, st) : v == 3 ? launch_tile_cfg<Tile7d>(a, st) : v == 2 ? launch_tile_cfg<Tile7c>(a, st) : v ? launch_tile_cfg<Tile7b>(a, st) : launch_tile_cfg<Tile7>(a, st);
   }
   return cudaErrorNotSupported;
 }
