@@ -85,6 +85,16 @@ csx_status ensure_device(csx_plan_s* p) {
     csx_status s = upload_pass(ps);
     if (s != CSX_OK) return s;
   }
+  {
+    cudaStream_t side;
+    cudaEvent_t a, b;
+    CSX_CUDA(cudaStreamCreateWithFlags(&side, cudaStreamNonBlocking), "side stream");
+    CSX_CUDA(cudaEventCreateWithFlags(&a, cudaEventDisableTiming), "event");
+    CSX_CUDA(cudaEventCreateWithFlags(&b, cudaEventDisableTiming), "event");
+    p->side = side;
+    p->ev_fork = a;
+    p->ev_join = b;
+  }
   CSX_CUDA(cudaMalloc(&p->d_wbase, p->w.size() * sizeof(double)), "cudaMalloc(w)");
   CSX_CUDA(cudaMemcpy(p->d_wbase, p->w.data(), p->w.size() * sizeof(double),
                       cudaMemcpyHostToDevice), "upload w");
@@ -112,6 +122,22 @@ csx_status ensure_grid(csx_plan_s* p, Padded* pd, double** bufs, const int64_t* 
 csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) {
   csx_engine eng = p->engine;
   cudaError_t e = cudaSuccess;
+  // TC_TILE 2D, FIXED, Tf > 1: the edge CTAs skip the band, so k_band (which writes only band
+  // points) runs on the side stream concurrently with the TC kernel; the caller's stream waits
+  // for it after the TC launch.
+  const bool band_side = eng == CSX_ENGINE_TC_TILE && p->bc == CSX_BC_FIXED && p->ndim == 2 &&
+                         ps.tf > 1 && c.part != 1;
+  if (band_side) {
+    cudaStream_t side = (cudaStream_t)p->side;
+    CSX_CUDA(cudaEventRecord((cudaEvent_t)p->ev_fork, st), "fork");
+    CSX_CUDA(cudaStreamWaitEvent(side, (cudaEvent_t)p->ev_fork, 0), "fork wait");
+    int launched = 0;
+    e = launch_band(p->ndim, p->radius, ps.tf, c.src, c.dst, c.E, c.gorg, p->E, p->w.data(), side,
+                    &launched);
+    if (e != cudaSuccess) return cuda_fail(e, "band fix-up launch");
+    p->n_launches += launched;
+    CSX_CUDA(cudaEventRecord((cudaEvent_t)p->ev_join, side), "join");
+  }
   if (eng == CSX_ENGINE_TC_S2R || eng == CSX_ENGINE_TC_TILE) {
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     const bool prof = p->prof && ps.tf == p->tf;  // time the main-pass (dominant) kernel only
@@ -186,6 +212,7 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
     if (ps.tf == p->tf) p->n_tc_launches += 1;
     p->n_launches += 1;
   }
+  if (band_side) CSX_CUDA(cudaStreamWaitEvent(st, (cudaEvent_t)p->ev_join, 0), "join wait");
   const bool direct_all = eng == CSX_ENGINE_DIRECT;
   const int real[3] = {p->ndim == 3, p->ndim >= 2, 1};
   if (eng == CSX_ENGINE_TC_TILE && c.part == 1) return CSX_OK;  // fix-ups run with the edge part
@@ -223,7 +250,7 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
       e = launch_frame_copy(c.src, c.dst, c.E, c.gorg, p->E, real, p->radius, st);
       if (e != cudaSuccess) return cuda_fail(e, "frame copy launch");
       p->n_launches += 1;
-    } else {
+    } else if (!band_side) {
       int launched = 0;
       e = launch_band(p->ndim, p->radius, ps.tf, c.src, c.dst, c.E, c.gorg, p->E, p->w.data(), st,
                       &launched);
@@ -422,6 +449,9 @@ csx_status csx_profile_read(csx_plan_t p, double* tc_ms, int64_t* tc_launches, i
 csx_status csx_plan_destroy(csx_plan_t p) {
   if (!p) return CSX_OK;
   for (void* ev : p->prof_events) cudaEventDestroy((cudaEvent_t)ev);
+  if (p->side) cudaStreamDestroy((cudaStream_t)p->side);
+  if (p->ev_fork) cudaEventDestroy((cudaEvent_t)p->ev_fork);
+  if (p->ev_join) cudaEventDestroy((cudaEvent_t)p->ev_join);
   if (p->device >= 0) {
     int cur = 0;
     cudaGetDevice(&cur);

@@ -111,6 +111,10 @@ struct csx_plan_s {
   int64_t s_lo = -1, s_hi = -1;
   int s_rank = -1, s_nranks = 0;
   double* d_dense = nullptr;       // csx_run_host staging grid
+  // side stream: the FIXED band fix-up of a TC_TILE 2D pass runs concurrently with the pass
+  void* side = nullptr;            // cudaStream_t
+  void* ev_fork = nullptr;         // cudaEvent_t
+  void* ev_join = nullptr;
   // measurement hooks
   bool prof = false;
   std::vector<void*> prof_events;  // cudaEvent_t pairs around TC launches
