@@ -335,7 +335,7 @@ struct Tile3DCfg {
   static constexpr int NCW = WM * WN;
   static constexpr int NT = 32 * (NCW + 1);
   static constexpr int SMEM = STAGES * STAGE * 8;
-  static_assert(STAGES >= NK + 2, "plane ring must hold the NK+1 planes of two outputs plus one in flight");
+  static_assert(STAGES >= NK + 1, "plane ring must hold NK planes plus one in flight");
 };
 
 template <class C>
@@ -404,29 +404,17 @@ __global__ void __launch_bounds__(C::NT, 2) k_tile3d(S2RArgs a, int tc_mask) {
       const int64_t qq = q0 + k;
       mbar_wait(&full[qq % C::STAGES], (uint32_t)((qq / C::STAGES) & 1));
     }
-    // Two output planes (zo, zo+1) per iteration: each staged plane's A fragments are loaded
-    // once and feed both planes' accumulators (twice the independent DMMA chains per warp).
-    for (int64_t zo = z0; zo < z1; zo += 2) {
-      const int npl = zo + 1 < z1 ? 2 : 1;
-      const int64_t qn = q0 + (zo - z0) + 2 * C::R + (npl - 1);  // newest plane zo + npl-1 + R
-      for (int64_t qq = q0 + (zo - z0) + 2 * C::R; qq <= qn; ++qq)
-        mbar_wait(&full[qq % C::STAGES], (uint32_t)((qq / C::STAGES) & 1));
-      double acc[2][C::G][2];
+    for (int64_t zo = z0; zo < z1; ++zo) {
+      const int64_t qn = q0 + (zo - z0) + 2 * C::R;  // newest plane zo + R
+      mbar_wait(&full[qn % C::STAGES], (uint32_t)((qn / C::STAGES) & 1));
+      double acc[C::G][2];
 #pragma unroll
-      for (int o = 0; o < 2; ++o)
+      for (int j = 0; j < C::G; ++j) acc[j][0] = acc[j][1] = 0.0;
 #pragma unroll
-        for (int j = 0; j < C::G; ++j) acc[o][j][0] = acc[o][j][1] = 0.0;
-      // staged plane k (k = 0 .. NK) is input plane zo - R + k; it feeds output zo with z offset
-      // dz = k (k < NK) and output zo+1 with dz = k - 1 (k >= 1)
-#pragma unroll
-      for (int k = 0; k <= C::NK; ++k) {
-        if (k == C::NK && npl == 1) break;
-        const int64_t qp = q0 + (zo - z0) + k;
+      for (int dz = 0; dz < C::NK; ++dz) {
+        const int64_t qp = q0 + (zo - z0) + dz;  // plane zo - R + dz
         const double* stg = smem + (qp % C::STAGES) * C::STAGE;
-        const int dz0 = k, dz1 = k - 1;
-        const bool tc0 = k < C::NK && (tc_mask & (1 << dz0));
-        const bool tc1 = npl == 2 && k >= 1 && (tc_mask & (1 << dz1));
-        if (tc0 || tc1) {
+        if (tc_mask & (1 << dz)) {
           const double* base = stg + (wm * C::A * C::G) * C::TP + wn * 8 * C::B + C::ODD + C::B * g + t;
 #pragma unroll
           for (int ra = 0; ra < C::A * C::G + C::NK - 1; ++ra) {
@@ -438,74 +426,59 @@ __global__ void __launch_bounds__(C::NT, 2) k_tile3d(S2RArgs a, int tc_mask) {
 #pragma unroll
               for (int j = 0; j < C::G; ++j) {
                 const int rho = ra - C::A * j;
-                if (rho >= 0 && rho < C::KR) {
-                  if (tc0) dmma_t(acc[0][j][0], acc[0][j][1], f[h], wf[k < C::NK ? dz0 : 0][rho * (C::KC / 4) + h]);
-                  if (tc1) dmma_t(acc[1][j][0], acc[1][j][1], f[h], wf[k >= 1 ? dz1 : 0][rho * (C::KC / 4) + h]);
-                }
+                if (rho >= 0 && rho < C::KR)
+                  dmma_t(acc[j][0], acc[j][1], f[h], wf[dz][rho * (C::KC / 4) + h]);
               }
           }
-        }
-        if (any_cuda) {
+        } else if (any_cuda && wz[dz] != 0.0) {
 #pragma unroll
           for (int j = 0; j < C::G; ++j) {
             const int lr = wm * C::A * C::G + C::A * j + alpha + C::R;
             const int lc = wn * 8 * C::B + C::B * g + beta + C::R + C::ODD;
             const double2 v = *reinterpret_cast<const double2*>(stg + lr * C::TP + lc);
-            if (k < C::NK && !tc0 && wz[k < C::NK ? dz0 : 0] != 0.0) {
-              acc[0][j][0] = fma(wz[dz0], v.x, acc[0][j][0]);
-              acc[0][j][1] = fma(wz[dz0], v.y, acc[0][j][1]);
-            }
-            if (npl == 2 && k >= 1 && !tc1 && wz[k >= 1 ? dz1 : 0] != 0.0) {
-              acc[1][j][0] = fma(wz[dz1], v.x, acc[1][j][0]);
-              acc[1][j][1] = fma(wz[dz1], v.y, acc[1][j][1]);
-            }
+            acc[j][0] = fma(wz[dz], v.x, acc[j][0]);
+            acc[j][1] = fma(wz[dz], v.y, acc[j][1]);
           }
         }
       }
-      for (int o = 0; o < npl; ++o) {
-        const int64_t zz = zo + o;
-        // FIXED frame (held points) of this output plane: the staged plane zz (k = R + o)
-        const int64_t gzo = zz + a.gorg0;
-        const bool plane_frame = a.hold_frame && (gzo < C::R || gzo >= a.GE0 - C::R);
-        const bool edge = a.hold_frame &&
-                          (plane_frame || (int64_t)ty * C::BM + a.gorg1 < C::R ||
-                           (int64_t)(ty + 1) * C::BM + a.gorg1 > a.GE1 - C::R ||
-                           (int64_t)tx * C::BN + a.gorg2 < C::R || (int64_t)(tx + 1) * C::BN + a.gorg2 > a.GE2 - C::R);
-        const double* cstg = smem + ((q0 + (zz - z0) + C::R) % C::STAGES) * C::STAGE;
-        double* plane = a.dst.p + zz * a.dst.s0;
+      // FIXED frame (held points) of this output plane: the staged plane zo (dz = R) holds them
+      const int64_t gzo = zo + a.gorg0;
+      const bool plane_frame = a.hold_frame && (gzo < C::R || gzo >= a.GE0 - C::R);
+      const bool edge = a.hold_frame &&
+                        (plane_frame || (int64_t)ty * C::BM + a.gorg1 < C::R ||
+                         (int64_t)(ty + 1) * C::BM + a.gorg1 > a.GE1 - C::R ||
+                         (int64_t)tx * C::BN + a.gorg2 < C::R || (int64_t)(tx + 1) * C::BN + a.gorg2 > a.GE2 - C::R);
+      const double* cstg = smem + ((q0 + (zo - z0) + C::R) % C::STAGES) * C::STAGE;
+      double* plane = a.dst.p + zo * a.dst.s0;
 #pragma unroll
-        for (int j = 0; j < C::G; ++j) {
-          const int64_t row = row0 + C::A * j;
-          if (row < a.E1 && col < a.E2) {
-            double* p = plane + row * a.dst.s1 + col;
-            const double v0 = o ? acc[1][j][0] : acc[0][j][0];
-            const double v1 = o ? acc[1][j][1] : acc[0][j][1];
-            if (!edge) {
-              if (col + 1 < a.E2 && ((reinterpret_cast<uintptr_t>(p) & 15) == 0)) {
-                *reinterpret_cast<double2*>(p) = make_double2(v0, v1);
-              } else {
-                p[0] = v0;
-                if (col + 1 < a.E2) p[1] = v1;
-              }
+      for (int j = 0; j < C::G; ++j) {
+        const int64_t row = row0 + C::A * j;
+        if (row < a.E1 && col < a.E2) {
+          double* p = plane + row * a.dst.s1 + col;
+          if (!edge) {
+            if (col + 1 < a.E2 && ((reinterpret_cast<uintptr_t>(p) & 15) == 0)) {
+              *reinterpret_cast<double2*>(p) = make_double2(acc[j][0], acc[j][1]);
             } else {
-              const int64_t grow = row + a.gorg1;
-              const bool rf = plane_frame || grow < C::R || grow >= a.GE1 - C::R;
+              p[0] = acc[j][0];
+              if (col + 1 < a.E2) p[1] = acc[j][1];
+            }
+          } else {
+            const int64_t grow = row + a.gorg1;
+            const bool rf = plane_frame || grow < C::R || grow >= a.GE1 - C::R;
 #pragma unroll
-              for (int e = 0; e < 2; ++e) {
-                const int64_t c = col + e, gc = c + a.gorg2;
-                if (c >= a.E2) continue;
-                double v = e ? v1 : v0;
-                if (rf || gc < C::R || gc >= a.GE2 - C::R)
-                  v = cstg[(int)(row - (int64_t)ty * C::BM + C::R) * C::TP + (int)(c - (int64_t)tx * C::BN) + C::R + C::ODD];
-                p[e] = v;
-              }
+            for (int e = 0; e < 2; ++e) {
+              const int64_t c = col + e, gc = c + a.gorg2;
+              if (c >= a.E2) continue;
+              double v = acc[j][e];
+              if (rf || gc < C::R || gc >= a.GE2 - C::R)
+                v = cstg[(int)(row - (int64_t)ty * C::BM + C::R) * C::TP + (int)(c - (int64_t)tx * C::BN) + C::R + C::ODD];
+              p[e] = v;
             }
           }
         }
       }
       __syncwarp();
-      if (lane == 0)
-        for (int o = 0; o < npl; ++o) mbar_arrive(&empty[(q0 + (zo - z0) + o) % C::STAGES]);  // planes zo-R+o done
+      if (lane == 0) mbar_arrive(&empty[(q0 + (zo - z0)) % C::STAGES]);  // plane zo-R is done
     }
     // release the last 2R planes of the item (not released by an output plane)
     __syncwarp();
