@@ -350,7 +350,7 @@ __device__ __forceinline__ void issue_plane(const S2RArgs& a, int ty, int tx, in
 }
 
 template <class C>
-__global__ void __launch_bounds__(C::NT, 2) k_tile3d(S2RArgs a, int tc_mask) {
+__global__ void __launch_bounds__(C::NT, (C::NCW > 8 ? 1 : 2)) k_tile3d(S2RArgs a, int tc_mask) {
   extern __shared__ __align__(128) double smem[];
   __shared__ __align__(8) uint64_t full[C::STAGES], empty[C::STAGES];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -488,7 +488,8 @@ __global__ void __launch_bounds__(C::NT, 2) k_tile3d(S2RArgs a, int tc_mask) {
   }
 }
 
-using Tile3D3 = Tile3DCfg<3, 8, 2, 2, 5, 32>;  // CTA 64 x 32 outputs, 4 DMMA warps, 4-plane ring, 32 planes per item
+using Tile3D3 = Tile3DCfg<3, 8, 2, 2, 5, 32>;  // CTA 64 x 32 outputs, 4 DMMA warps, 5-plane ring, 32 planes per item
+using Tile3D3b = Tile3DCfg<3, 4, 4, 4, 4, 32>;  // CTA 64 x 64 outputs, 16 DMMA warps, 1 CTA/SM
 
 
 // ------------------------------------------------------------------------------------------
@@ -668,14 +669,15 @@ static cudaError_t launch_tile1d_cfg(S2RArgs a, cudaStream_t st) {
   return cudaGetLastError();
 }
 
+// consumer warps / stages per nk as measured on B200 (Heat-1D nk=15: 8 warps, 1D5P nk=13: 4)
 static cudaError_t launch_tile1d(int nk, const S2RArgs& a, cudaStream_t st) {
   switch (nk) {
-    case 3: return launch_tile1d_cfg<Tile1DCfg<3, 256, 8, 5>>(a, st);
-    case 5: return launch_tile1d_cfg<Tile1DCfg<5, 252, 8, 5>>(a, st);
-    case 7: return launch_tile1d_cfg<Tile1DCfg<7, 256, 8, 5>>(a, st);
-    case 9: return launch_tile1d_cfg<Tile1DCfg<9, 250, 8, 5>>(a, st);
-    case 11: return launch_tile1d_cfg<Tile1DCfg<11, 252, 8, 5>>(a, st);
-    case 13: return launch_tile1d_cfg<Tile1DCfg<13, 252, 8, 5>>(a, st);
+    case 3: return launch_tile1d_cfg<Tile1DCfg<3, 256, 4, 6>>(a, st);
+    case 5: return launch_tile1d_cfg<Tile1DCfg<5, 252, 4, 6>>(a, st);
+    case 7: return launch_tile1d_cfg<Tile1DCfg<7, 256, 4, 6>>(a, st);
+    case 9: return launch_tile1d_cfg<Tile1DCfg<9, 250, 4, 6>>(a, st);
+    case 11: return launch_tile1d_cfg<Tile1DCfg<11, 252, 4, 6>>(a, st);
+    case 13: return launch_tile1d_cfg<Tile1DCfg<13, 252, 4, 6>>(a, st);
     case 15: return launch_tile1d_cfg<Tile1DCfg<15, 256, 8, 5>>(a, st);
   }
   return cudaErrorNotSupported;
@@ -724,7 +726,11 @@ static cudaError_t launch_tile3d_cfg(S2RArgs a, int tc_mask, cudaStream_t st) {
 cudaError_t launch_tile(int ndim, int nk, const S2RArgs& a, cudaStream_t st) {
   if (ndim == 1) return launch_tile1d(nk, a, st);
   if (ndim == 3) {
-    if (nk == 3) return launch_tile3d_cfg<Tile3D3>(a, a.tc_mask, st);
+    if (nk == 3) {
+      const char* e = getenv("CSX_TILE3D_VARIANT");
+      if (e && e[0] == '1') return launch_tile3d_cfg<Tile3D3b>(a, a.tc_mask, st);
+      return launch_tile3d_cfg<Tile3D3>(a, a.tc_mask, st);
+    }
     return cudaErrorNotSupported;
   }
   if (ndim != 2) return cudaErrorNotSupported;
