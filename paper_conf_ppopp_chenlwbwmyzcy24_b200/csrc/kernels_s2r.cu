@@ -146,24 +146,27 @@ __global__ void __launch_bounds__(S2R2D<NK>::NT, 2) k_s2r2d(S2RArgs a) {
     if (lane == 0) s2r_mbar_arrive(&empty[s]);  // raw stage consumed
     asm volatile("bar.sync 1, %0;\n" ::"r"(NC) : "memory");  // A/B complete
     const int64_t col = (int64_t)tx * G::BN + g * G::SW + 2 * t;
-#pragma unroll 1
-    for (int xr = warp * (G::BM / G::NCW); xr < (warp + 1) * (G::BM / G::NCW); xr += 2) {
-      const double* pa = sA + g * G::PITCH + G::NKV * xr + t;
-      const double* pb = sB + g * G::PITCH + G::NKV * xr + t;
-      double c00 = 0.0, c01 = 0.0, c10 = 0.0, c11 = 0.0;
+    // the warp's BM/NCW = 4 output rows as 4 independent accumulation chains (vitrolite B
+    // accumulated onto A, P.1332-1336)
+    constexpr int RW = G::BM / G::NCW;
+    const int xr0 = warp * RW;
+    const double* pa = sA + g * G::PITCH + G::NKV * xr0 + t;
+    const double* pb = sB + g * G::PITCH + G::NKV * xr0 + t;
+    double c[RW][2];
 #pragma unroll
-      for (int s2 = 0; s2 < G::KS; ++s2) {
-        dmma(c00, c01, pa[4 * s2], wa[s2]);
-        dmma(c10, c11, pa[4 * s2 + G::NKV], wa[s2]);
-      }
+    for (int q = 0; q < RW; ++q) c[q][0] = c[q][1] = 0.0;
 #pragma unroll
-      for (int s2 = 0; s2 < G::KS; ++s2) {
-        dmma(c00, c01, pb[4 * s2], wb[s2]);
-        dmma(c10, c11, pb[4 * s2 + G::NKV], wb[s2]);
-      }
-      const int64_t row = (int64_t)ty * G::BM + xr;
-      if (row < a.E1) store_pair(a.dst.p + row * a.dst.s1, col, a.E2, v0, v1, c00, c01);
-      if (row + 1 < a.E1) store_pair(a.dst.p + (row + 1) * a.dst.s1, col, a.E2, v0, v1, c10, c11);
+    for (int s2 = 0; s2 < G::KS; ++s2)
+#pragma unroll
+      for (int q = 0; q < RW; ++q) dmma(c[q][0], c[q][1], pa[4 * s2 + q * G::NKV], wa[s2]);
+#pragma unroll
+    for (int s2 = 0; s2 < G::KS; ++s2)
+#pragma unroll
+      for (int q = 0; q < RW; ++q) dmma(c[q][0], c[q][1], pb[4 * s2 + q * G::NKV], wb[s2]);
+#pragma unroll
+    for (int q = 0; q < RW; ++q) {
+      const int64_t row = (int64_t)ty * G::BM + xr0 + q;
+      if (row < a.E1) store_pair(a.dst.p + row * a.dst.s1, col, a.E2, v0, v1, c[q][0], c[q][1]);
     }
   }
 }

