@@ -45,6 +45,8 @@ CONFIGS = {
     "heat1d_10240000": ("heat1d", (10240000,), 1000, "fixed", 0),        # extra (north-star list)
     "1d5p_10240000": ("1d5p", (10240000,), 1000, "fixed", 0),
     "heat2d_10240": ("heat2d", (10240, 10240), 100, "fixed", 0),
+    "star2d9p_10240": ("star2d9p", (10240, 10240), 100, "fixed", 0),     # Table 3 extra shapes
+    "box2d25p_10240": ("box2d25p", (10240, 10240), 100, "fixed", 0),
 }
 DEFAULT = "box2d9p_10240"
 METRIC = "FP64 GStencils/s"

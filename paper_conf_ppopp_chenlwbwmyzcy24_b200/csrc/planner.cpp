@@ -116,7 +116,7 @@ void layout_padded(const csx_plan_s* p, const int64_t* E, Padded* pd) {
   pd->O[1] = real1 ? H : 0;
   pd->O[2] = 16 * ((H + 15) / 16);  // >= H, interior rows 128-byte aligned
   if (pd->O[2] < 16) pd->O[2] = 16;
-  pd->A[0] = real0 ? (E[0] + 2 * H + 2) : 1;
+  pd->A[0] = real0 ? (E[0] + 2 * H + 16) : 1;  // direct-kernel z tiles (8) overhang the last plane
   pd->A[1] = real1 ? (pd->O[1] + E[1] + 128 + H + 2) : 1;
   const int64_t need2 = pd->O[2] + E[2] + 160 + H + 32;
   pd->A[2] = 32 * ((need2 + (p->ndim == 1 ? 2048 : 0) + 31) / 32);  // 1D tiles overhang more
