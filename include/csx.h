@@ -83,7 +83,8 @@ csx_status csx_plan_set_engine(csx_plan_t plan, csx_engine engine);
 /* TC_S2R breakdown variants (Fig 6, P.1865-1950), 2D only: padding = 0 uses the bare
  * stencil2row pitch nk*rr (Fig 5's conflicting 266) instead of the conflict-free one (268);
  * dirty_bits = 0 replaces the dirty-bits padding by conditional stores in the LUT copy loop.
- * (1, 1) is the paper's full design (the default); (0, 0) = variant III, (1, 0) = IV. */
+ * (1, 1) is the paper's full design (the default); (0, 0) = variant III, (1, 0) = IV;
+ * padding = 2 selects variant II (same tiles, the tessellation GEMM on CUDA cores / DFMA). */
 csx_status csx_plan_set_s2r_variant(csx_plan_t plan, int padding, int dirty_bits);
 
 /* Advance d_in by `timesteps` base steps into d_out (both prod(extents) doubles, device,

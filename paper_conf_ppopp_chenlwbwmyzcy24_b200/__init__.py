@@ -139,9 +139,10 @@ def csx_plan_set_engine(plan, engine: int):
     _check(_lib.csx_plan_set_engine(plan, int(engine)), "csx_plan_set_engine")
 
 
-def csx_plan_set_s2r_variant(plan, padding: bool = True, dirty_bits: bool = True):
-    _check(_lib.csx_plan_set_s2r_variant(plan, int(bool(padding)), int(bool(dirty_bits))),
-           "csx_plan_set_s2r_variant")
+def csx_plan_set_s2r_variant(plan, padding=True, dirty_bits: bool = True):
+    """padding: True/False, or 2 for breakdown variant II (CUDA-core tessellation)."""
+    _check(_lib.csx_plan_set_s2r_variant(plan, 2 if padding == 2 else int(bool(padding)),
+                                         int(bool(dirty_bits))), "csx_plan_set_s2r_variant")
 
 
 def csx_run(plan, d_in, d_out, timesteps: int, n: int, stream=None):
@@ -292,7 +293,7 @@ class Plan:
     def handle(self):
         return self._h
 
-    def set_s2r_variant(self, padding: bool = True, dirty_bits: bool = True):
+    def set_s2r_variant(self, padding=True, dirty_bits: bool = True):
         csx_plan_set_s2r_variant(self._h, padding, dirty_bits)
 
     def set_engine(self, engine: str):

@@ -189,7 +189,7 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
       e = launch_tile(p->ndim, ps.nk, a, st);
     } else {
       a.frags = ps.d_frags;
-      a.s2r_variant = (p->s2r_pad ? 1 : 0) | (p->s2r_dirty ? 2 : 0);
+      a.s2r_variant = (p->s2r_pad ? 1 : 0) | (p->s2r_dirty ? 2 : 0) | (p->s2r_fma ? 4 : 0);
       int tc_mask = 0;
       if (p->ndim == 1) {
         a.tiles_x = (int)((c.E[2] + ps.bn - 1) / ps.bn);
@@ -340,6 +340,9 @@ csx_status csx_plan(int ndim, const int64_t* extents, csx_shape shape, int radiu
 
 csx_status csx_plan_set_s2r_variant(csx_plan_t p, int padding, int dirty_bits) {
   if (!p) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL plan");
+  // padding = 2: breakdown variant II (padding + dirty bits, tessellation on CUDA cores)
+  p->s2r_fma = padding == 2;
+  if (p->s2r_fma) { padding = 1; dirty_bits = 1; }
   if (p->ndim != 2 && !(padding && dirty_bits))
     return fail(CSX_ERR_UNSUPPORTED, "breakdown variants are 2D only");
   p->s2r_pad = padding != 0;

@@ -97,6 +97,7 @@ struct csx_plan_s {
   csx_engine engine_req = CSX_ENGINE_AUTO;
   bool s2r_pad = true;             // TC_S2R 2D: conflict-free pitch (Fig 5)
   bool s2r_dirty = true;           // TC_S2R 2D: dirty-bits padding instead of branches
+  bool s2r_fma = false;            // TC_S2R 2D: breakdown II, tessellation on CUDA cores
   csx_engine engine = CSX_ENGINE_TC_S2R;
   std::vector<csx::Pass> passes;   // index tf' - 1, for tf' = 1..tf
   // device state (allocated at the first run)

@@ -75,10 +75,13 @@ __device__ __forceinline__ void s2r_issue_rows(const double* src, int64_t pitch,
         : "memory");
 }
 
-template <int NK, bool PAD, bool DIRTY>
+// FMA = true is breakdown variant II (Fig 6): the same implicit stencil2row tiles, the dual
+// tessellation computed on CUDA cores (DFMA) from weight matrices staged in shared memory.
+template <int NK, bool PAD, bool DIRTY, bool FMA = false>
 __global__ void __launch_bounds__(S2R2D<NK>::NT, 2) k_s2r2d(S2RArgs a) {
   using G = S2R2D<NK, PAD>;
   extern __shared__ __align__(128) double smem[];
+  __shared__ double sW[FMA ? 2 * G::KS * 4 * 8 : 1];  // [A|B][k][c] for the FMA variant
   __shared__ __align__(8) uint64_t full[G::RAW_STAGES], empty[G::RAW_STAGES];
   double* raw = smem;                                           // RAW_STAGES x RAW
   double* sA = raw + G::RAW_STAGES * G::RAW;
@@ -90,6 +93,11 @@ __global__ void __launch_bounds__(S2R2D<NK>::NT, 2) k_s2r2d(S2RArgs a) {
   // the LUT packs the A and B offsets of each region element (P.1711-1721).
   for (int i = tid; i < 2 * (G::STRIPS + 1) * G::PITCH; i += G::NT) sA[i] = 0.0;
   for (int i = tid; i < G::NE; i += G::NT) sL[i] = (uint32_t)a.lut[i].y;
+  if (FMA)  // W[k][c] from the per-lane fragments: lane l of slice s holds W[4s + l%4][l/4]
+    for (int i = tid; i < 2 * G::KS * 32; i += G::NT) {
+      const int m = i / (G::KS * 32), r = i - m * G::KS * 32, k = r / 8, c = r % 8;
+      sW[i] = a.frags[(m * G::KS + k / 4) * 32 + (k % 4) + 4 * c];
+    }
   if (tid == 0) {
     for (int s = 0; s < G::RAW_STAGES; ++s) {
       s2r_mbar_init(&full[s], 1);
@@ -155,14 +163,31 @@ __global__ void __launch_bounds__(S2R2D<NK>::NT, 2) k_s2r2d(S2RArgs a) {
     double c[RW][2];
 #pragma unroll
     for (int q = 0; q < RW; ++q) c[q][0] = c[q][1] = 0.0;
+    if (!FMA) {
 #pragma unroll
-    for (int s2 = 0; s2 < G::KS; ++s2)
+      for (int s2 = 0; s2 < G::KS; ++s2)
 #pragma unroll
-      for (int q = 0; q < RW; ++q) dmma(c[q][0], c[q][1], pa[4 * s2 + q * G::NKV], wa[s2]);
+        for (int q = 0; q < RW; ++q) dmma(c[q][0], c[q][1], pa[4 * s2 + q * G::NKV], wa[s2]);
 #pragma unroll
-    for (int s2 = 0; s2 < G::KS; ++s2)
+      for (int s2 = 0; s2 < G::KS; ++s2)
 #pragma unroll
-      for (int q = 0; q < RW; ++q) dmma(c[q][0], c[q][1], pb[4 * s2 + q * G::NKV], wb[s2]);
+        for (int q = 0; q < RW; ++q) dmma(c[q][0], c[q][1], pb[4 * s2 + q * G::NKV], wb[s2]);
+    } else {
+      // lane (g, t) owns C[g][2t], C[g][2t+1]: sum over k of tile[g][k] * W[k][c]
+      const double* qa = sA + g * G::PITCH + G::NKV * xr0;
+      const double* qb = sB + g * G::PITCH + G::NKV * xr0;
+#pragma unroll 4
+      for (int k = 0; k < G::NKV * G::NKV; ++k) {
+        const double2 wA = *reinterpret_cast<const double2*>(&sW[k * 8 + 2 * t]);
+        const double2 wB = *reinterpret_cast<const double2*>(&sW[G::KS * 32 + k * 8 + 2 * t]);
+#pragma unroll
+        for (int q = 0; q < RW; ++q) {
+          const double xa = qa[k + q * G::NKV], xb = qb[k + q * G::NKV];
+          c[q][0] = fma(xa, wA.x, fma(xb, wB.x, c[q][0]));
+          c[q][1] = fma(xa, wA.y, fma(xb, wB.y, c[q][1]));
+        }
+      }
+    }
 #pragma unroll
     for (int q = 0; q < RW; ++q) {
       const int64_t row = (int64_t)ty * G::BM + xr0 + q;
@@ -366,7 +391,10 @@ static cudaError_t launch_persistent(K kernel, int smem, int nthreads, int64_t i
 
 template <int NK>
 static cudaError_t launch_s2r2d_var(const S2RArgs& a, int variant, cudaStream_t st) {
-  // variant bit 0 = padding, bit 1 = dirty bits (default 3 = the paper's full design)
+  // variant bit 0 = padding, bit 1 = dirty bits (default 3 = the paper's full design),
+  // bit 2 = CUDA-core tessellation (breakdown II, with padding and dirty bits)
+  if (variant & 4)
+    return launch_persistent(k_s2r2d<NK, true, true, true>, S2R2D<NK, true>::SMEM, S2R2D<NK>::NT, a.ntiles, st, a);
   switch (variant) {
     case 3: return launch_persistent(k_s2r2d<NK, true, true>, S2R2D<NK, true>::SMEM, S2R2D<NK>::NT, a.ntiles, st, a);
     case 1: return launch_persistent(k_s2r2d<NK, true, false>, S2R2D<NK, true>::SMEM, S2R2D<NK>::NT, a.ntiles, st, a);

@@ -350,7 +350,7 @@ __device__ __forceinline__ void issue_plane(const S2RArgs& a, int ty, int tx, in
 }
 
 template <class C>
-__global__ void __launch_bounds__(C::NT, (C::NCW > 8 ? 1 : 2)) k_tile3d(S2RArgs a, int tc_mask) {
+__global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2)) k_tile3d(S2RArgs a, int tc_mask) {
   extern __shared__ __align__(128) double smem[];
   __shared__ __align__(8) uint64_t full[C::STAGES], empty[C::STAGES];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -490,6 +490,7 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 8 ? 1 : 2)) k_tile3d(S2RArgs 
 
 using Tile3D3 = Tile3DCfg<3, 8, 2, 2, 5, 32>;  // CTA 64 x 32 outputs, 4 DMMA warps, 5-plane ring, 32 planes per item
 using Tile3D3b = Tile3DCfg<3, 4, 4, 4, 4, 32>;  // CTA 64 x 64 outputs, 16 DMMA warps, 1 CTA/SM
+using Tile3D3c = Tile3DCfg<3, 8, 2, 4, 6, 32>;  // CTA 64 x 64 outputs, 8 DMMA warps, 6-plane ring
 
 
 // ------------------------------------------------------------------------------------------
@@ -729,6 +730,7 @@ cudaError_t launch_tile(int ndim, int nk, const S2RArgs& a, cudaStream_t st) {
     if (nk == 3) {
       const char* e = getenv("CSX_TILE3D_VARIANT");
       if (e && e[0] == '1') return launch_tile3d_cfg<Tile3D3b>(a, a.tc_mask, st);
+      if (e && e[0] == '2') return launch_tile3d_cfg<Tile3D3c>(a, a.tc_mask, st);
       return launch_tile3d_cfg<Tile3D3>(a, a.tc_mask, st);
     }
     return cudaErrorNotSupported;

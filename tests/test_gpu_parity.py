@@ -202,7 +202,7 @@ def test_direct_comparator_2d_all_radii(csx):
             assert rel(got, oracle.run(u0, w, bc, 9)) <= TOL, (r, tf, bc)
 
 
-@pytest.mark.parametrize("pad,dirty", [(0, 0), (1, 0), (0, 1), (1, 1)])
+@pytest.mark.parametrize("pad,dirty", [(0, 0), (1, 0), (0, 1), (1, 1), (2, 1)])
 def test_s2r_breakdown_variants(csx, pad, dirty):
     """Fig 6 breakdown variants of TC_S2R (no padding / no dirty bits) compute the same result."""
     for name in ("box2d9p", "heat2d", "box2d49p"):
@@ -210,7 +210,7 @@ def test_s2r_breakdown_variants(csx, pad, dirty):
         w = synth.random_weights(name)
         u0 = synth.grid((99, 140), seed=51)
         p = csx.Plan(u0.shape, w, shape=s.kind, bc="fixed", engine="tc_s2r")
-        p.set_s2r_variant(bool(pad), bool(dirty))
+        p.set_s2r_variant(2 if pad == 2 else bool(pad), bool(dirty))
         d_in = torch.from_numpy(u0).cuda()
         d_out = torch.empty_like(d_in)
         p.run(d_in, d_out, 7)
