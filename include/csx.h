@@ -150,10 +150,13 @@ typedef struct {
 csx_status csx_plan_info(const csx_plan_t plan, csx_plan_info_t* info);
 
 /* ----- Measurement hooks (bench.py) -----------------------------------------------------
- * With profiling enabled, every TC pass kernel launch (the dominant kernel) is bracketed by
- * CUDA events recorded on the launching stream, and every kernel the library launches is
- * counted.  csx_profile_read synchronises on the recorded events and returns the summed TC
- * kernel time (ms) and launch counts since the last reset. */
+ * csx_profile_enable(plan, n): n = 0 disables; n >= 1 brackets every n-th main-pass TC kernel
+ * launch (the dominant kernel) with CUDA events recorded on the launching stream (n = 1: all
+ * of them; events between launches defeat programmatic dependent launch, so a period > 1
+ * keeps most passes chained), and counts every kernel the library launches.  n < 0 ->
+ * CSX_ERR_INVALID_ARGUMENT.  csx_profile_read synchronises on the recorded events and returns
+ * the mean timed TC kernel duration x the number of main-pass TC launches (ms; = the summed
+ * time when n = 1) and the launch counts since the last reset. */
 csx_status csx_profile_enable(csx_plan_t plan, int enable);
 csx_status csx_profile_read(csx_plan_t plan, double* tc_kernel_ms, int64_t* tc_launches,
                             int64_t* total_launches, int reset);

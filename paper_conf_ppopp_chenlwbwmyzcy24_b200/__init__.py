@@ -217,8 +217,9 @@ def csx_plan_lut(plan):
     return a.reshape(rr.value, rc.value), b.reshape(rr.value, rc.value)
 
 
-def csx_profile_enable(plan, enable: bool = True):
-    _check(_lib.csx_profile_enable(plan, int(bool(enable))), "csx_profile_enable")
+def csx_profile_enable(plan, enable=True):
+    """enable: False/0 off, True/1 time every main-pass TC launch, n > 1 every n-th."""
+    _check(_lib.csx_profile_enable(plan, int(enable)), "csx_profile_enable")
 
 
 def csx_profile_read(plan, reset: bool = True):

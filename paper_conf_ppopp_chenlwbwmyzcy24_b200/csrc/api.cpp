@@ -140,7 +140,9 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
   }
   if (eng == CSX_ENGINE_TC_S2R || eng == CSX_ENGINE_TC_TILE) {
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
-    const bool prof = p->prof && ps.tf == p->tf;  // time the main-pass (dominant) kernel only
+    // time the main-pass (dominant) kernel only, every prof-th launch (events between kernels
+    // break programmatic dependent launch, so bench.py samples rather than brackets them all)
+    const bool prof = p->prof > 0 && ps.tf == p->tf && (p->n_tc_launches % p->prof) == 0;
     if (prof) {
       if (p->prof_used + 2 > p->prof_events.size()) {
         for (int k = 0; k < 64; ++k) {
@@ -163,6 +165,7 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
     a.wc = ps.d_wc;
     if (eng == CSX_ENGINE_TC_TILE) {
       a.frags = ps.d_tile_frags;
+      a.pdl = !band_side && c.part == 0;  // no PDL across the band join / halo-exchange waits
       if (p->ndim == 3)
         for (int dz = 0; dz < ps.nk; ++dz) a.tc_mask |= ps.plane_is_tc[dz] << dz;
       if (p->bc == CSX_BC_FIXED && p->ndim == 1) {  // 1D band recomputed in-kernel
@@ -423,7 +426,8 @@ csx_status csx_run_host(csx_plan_t p, const double* h_in, double* h_out, int64_t
 
 csx_status csx_profile_enable(csx_plan_t p, int enable) {
   if (!p) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL plan");
-  p->prof = enable != 0;
+  if (enable < 0) return fail(CSX_ERR_INVALID_ARGUMENT, "profile period must be >= 0");
+  p->prof = enable;
   return CSX_OK;
 }
 
@@ -431,14 +435,16 @@ csx_status csx_profile_read(csx_plan_t p, double* tc_ms, int64_t* tc_launches, i
                             int reset) {
   if (!p) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL plan");
   double ms = 0.0;
-  for (size_t i = 0; i + 1 < p->prof_used; i += 2) {
+  int64_t timed = 0;
+  for (size_t i = 0; i + 1 < p->prof_used; i += 2, ++timed) {
     cudaEvent_t a = (cudaEvent_t)p->prof_events[i], b = (cudaEvent_t)p->prof_events[i + 1];
     CSX_CUDA(cudaEventSynchronize(b), "cudaEventSynchronize");
     float f = 0.f;
     CSX_CUDA(cudaEventElapsedTime(&f, a, b), "cudaEventElapsedTime");
     ms += f;
   }
-  if (tc_ms) *tc_ms = ms;
+  // sampled launches: scale the mean timed duration to every main-pass launch
+  if (tc_ms) *tc_ms = timed > 0 ? ms / (double)timed * (double)p->n_tc_launches : 0.0;
   if (tc_launches) *tc_launches = p->n_tc_launches;
   if (total) *total = p->n_launches;
   if (reset) {

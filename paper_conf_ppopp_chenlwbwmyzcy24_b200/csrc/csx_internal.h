@@ -117,7 +117,7 @@ struct csx_plan_s {
   void* ev_fork = nullptr;         // cudaEvent_t
   void* ev_join = nullptr;
   // measurement hooks
-  bool prof = false;
+  int prof = 0;  // 0 off, n: time every n-th main-pass TC launch
   std::vector<void*> prof_events;  // cudaEvent_t pairs around TC launches
   size_t prof_used = 0;
   int64_t n_tc_launches = 0, n_launches = 0;

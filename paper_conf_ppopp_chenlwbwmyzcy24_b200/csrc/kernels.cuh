@@ -35,6 +35,7 @@ struct S2RArgs {
   int64_t ra0 = 0, ra1 = 0, rb0 = 0, rb1 = 0;  // slab-tile ranges, filled by the launcher
   int s2r_variant = 3;            // TC_S2R 2D: bit 0 padding, bit 1 dirty bits (breakdown)
   int fix_band = 0;
+  int pdl = 1;                    // TC_TILE: launch with programmatic dependent launch
   int hold_frame = 0;             // write held (frame) values from the staged tile (Tf = 1)
   int r = 0;
   const double* wbase = nullptr;  // base weights (2r+1)^2

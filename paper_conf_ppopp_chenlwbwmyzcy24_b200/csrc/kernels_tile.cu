@@ -63,6 +63,16 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
       : "memory");
 }
 
+// Programmatic dependent launch (sm_90+): the kernels below are launched with programmatic
+// stream serialisation (launch_pdl), so pass p+1's CTAs are scheduled onto SMs as pass p's CTAs
+// retire.  Everything before pdl_begin() touches only smem and the plan's constant tables;
+// griddepcontrol.wait then blocks until the previous grid has completed and its writes are
+// visible, so no global read of src (or write of dst, which the previous pass read) precedes it.
+__device__ __forceinline__ void pdl_begin() {
+  asm volatile("griddepcontrol.launch_dependents;\n" ::: "memory");
+  asm volatile("griddepcontrol.wait;\n" ::: "memory");
+}
+
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(bar)) : "memory");
 }
@@ -94,6 +104,31 @@ static int64_t set_ranges(S2RArgs& a, int64_t n, int64_t size, int64_t El, int R
     a.rb1 = n;
   }
   return (a.ra1 - a.ra0) + (a.rb1 - a.rb0);
+}
+
+static bool pdl_enabled() {
+  static const int v = [] {
+    const char* e = getenv("CSX_PDL");
+    return e ? atoi(e) : 1;
+  }();
+  return v != 0;
+}
+
+// launch with programmatic stream serialisation (see pdl_begin)
+template <class... KArgs, class... Args>
+static cudaError_t launch_pdl(bool pdl, void (*k)(KArgs...), int64_t grid, int nt, int smem,
+                              cudaStream_t st, Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3((unsigned)nt);
+  cfg.dynamicSmemBytes = (size_t)smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl && pdl_enabled() ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, k, args...);
 }
 
 static int64_t cap_grid(const S2RArgs& a, int64_t grid) {
@@ -166,6 +201,7 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_tile2d(S2RArgs a) {
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
   }
   __syncthreads();
+  pdl_begin();  // PDL: let the next pass launch; wait for the previous pass's writes
   if (warp == C::NCW) {
     // ---------------- producer ----------------
     int it = 0;
@@ -362,6 +398,7 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2)) k_tile3d(S2RArgs 
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
   }
   __syncthreads();
+  pdl_begin();  // PDL: let the next pass launch; wait for the previous pass's writes
   const int64_t ncol = (int64_t)a.tiles_x * a.tiles_y;
   if (warp == C::NCW) {  // producer: planes of every work item, in consumption order
     int64_t q = 0;
@@ -531,6 +568,7 @@ __global__ void __launch_bounds__(C::NT, 2) k_tile1d(S2RArgs a) {  // 2 CTAs/SM
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
   }
   __syncthreads();
+  pdl_begin();  // PDL: let the next pass launch; wait for the previous pass's writes
   if (warp == C::NCW) {  // producer: 8 segment copies per tile
     int it = 0;
     for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
@@ -666,8 +704,7 @@ static cudaError_t launch_tile1d_cfg(S2RArgs a, cudaStream_t st) {
   if (e != cudaSuccess) return e;
   int64_t grid = cap_grid(a, (int64_t)(occ < 1 ? 1 : occ) * num_sms());
   if (grid > a.ntiles) grid = a.ntiles;
-  k_tile1d<C><<<(unsigned)grid, C::NT, C::SMEM, st>>>(a);
-  return cudaGetLastError();
+  return launch_pdl(a.pdl != 0, k_tile1d<C>, grid, C::NT, C::SMEM, st, a);
 }
 
 // consumer warps / stages per nk as measured on B200 (Heat-1D nk=15: 8 warps, 1D5P nk=13: 4)
@@ -703,8 +740,7 @@ static cudaError_t launch_tile_cfg(S2RArgs a, cudaStream_t st) {
   if (e != cudaSuccess) return e;
   int64_t grid = cap_grid(a, (int64_t)(occ < 1 ? 1 : occ) * num_sms());
   if (grid > a.ntiles) grid = a.ntiles;
-  k_tile2d<C><<<(unsigned)grid, C::NT, C::SMEM, st>>>(a);
-  return cudaGetLastError();
+  return launch_pdl(a.pdl != 0, k_tile2d<C>, grid, C::NT, C::SMEM, st, a);
 }
 
 template <class C>
@@ -720,8 +756,7 @@ static cudaError_t launch_tile3d_cfg(S2RArgs a, int tc_mask, cudaStream_t st) {
   if (e != cudaSuccess) return e;
   int64_t grid = cap_grid(a, (int64_t)(occ < 1 ? 1 : occ) * num_sms());
   if (grid > a.ntiles) grid = a.ntiles;
-  k_tile3d<C><<<(unsigned)grid, C::NT, C::SMEM, st>>>(a, tc_mask);
-  return cudaGetLastError();
+  return launch_pdl(a.pdl != 0, k_tile3d<C>, grid, C::NT, C::SMEM, st, a, tc_mask);
 }
 
 cudaError_t launch_tile(int ndim, int nk, const S2RArgs& a, cudaStream_t st) {
