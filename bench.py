@@ -134,8 +134,11 @@ class ClockSampler:
 
 def algorithmic_mma(ndim, nk, engine, points, tc_planes):
     """DMMA.8x8x4 per pass over `points` outputs: Eq 13 generalised by
-    reading A7 (N fragments) and 3D planes for TC_S2R; 4x2/2x4 blocks for TC_TILE."""
-    if engine == "tc_s2r" or (engine == "tc_tile" and ndim == 1):
+    reading A7 (N fragments) and 3D planes for TC_S2R; 4x2/2x4 blocks for TC_TILE 2D/3D and
+    8-output Toeplitz blocks (K = nk + 7 rounded up to 4) for TC_TILE 1D."""
+    if engine == "tc_tile" and ndim == 1:
+        return points / 64 * math.ceil((nk + 7) / 4)
+    if engine == "tc_s2r":
         sw = nk + 1
         nf = (sw + 7) // 8
         k = nk if ndim == 1 else nk * nk

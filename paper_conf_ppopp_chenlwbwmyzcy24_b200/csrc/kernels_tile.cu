@@ -531,28 +531,34 @@ using Tile3D3c = Tile3DCfg<3, 8, 2, 4, 6, 32>;  // CTA 64 x 64 outputs, 8 DMMA w
 
 
 // ------------------------------------------------------------------------------------------
-// 1D (P.1779-1786) on the TC_TILE pipeline.  The paper's 1D dual tessellation is kept exactly —
-// strip k of a segment holds outputs [k(nk+1), (k+1)(nk+1)), Tile_A row = the nk inputs of the
-// strip, Tile_B row = the next nk, W_A / W_B as in 2D, N fragments for nk+1 > 8 (reading A7) —
-// but the 8 M rows of a DMMA are 8 different SEGMENTS of the tile, staged by cp.async.bulk with
-// a segment pitch P = 4 or 12 (mod 16) doubles.  The A/B fragments are then strided views of
-// the staged input (conflict-free, no LUT scatter), and the kernel streams HBM through a
-// STAGES-deep ring (the 1D path is HBM-bound: 16/Tf bytes per point-step).
-template <int NK_, int L_, int NCW_, int STAGES_>
+// 1D (P.1779-1786) on the TC_TILE pipeline, re-laid out for DMMA.8x8x4.  The 8 M rows of a DMMA
+// are 8 SEGMENTS of the tile (each L outputs, staged by cp.async.bulk with a segment pitch
+// P = 4 or 12 mod 16 doubles: conflict-free fragment loads); the 8 N columns are 8 CONSECUTIVE
+// outputs of a segment, so the weight operand is the banded Toeplitz matrix
+// W[k][n] = w[k - n] (0 <= k - n < nk) of K = nk + 7 rounded up to 4 rows — ks = ceil((nk+7)/4)
+// DMMAs per 8 x 8 outputs instead of the paper's 2 ceil(nk/4) nf per 8 x (nk+1) (6 vs 8 per 64
+// outputs at nk = 15, 5 vs 9.1 at nk = 13).  Block b+1's window is block b's shifted by 8
+// inputs = 2 k-slices, so an A fragment loaded from smem serves ks/2 blocks: a warp runs NB
+// blocks at once over a register window of 2 NB + ks - 2 fragments (0.5 LDS.64 per DMMA at
+// NB = 4, nk = 15).  The kernel streams HBM through a STAGES-deep ring.
+template <int NK_, int L_, int NCW_, int STAGES_, int NB_>
 struct Tile1DCfg {
-  static constexpr int NK = NK_, L = L_, NCW = NCW_, STAGES = STAGES_;
-  static constexpr int SW = NK + 1;
-  static constexpr int NF = (SW + 7) / 8;
-  static constexpr int KA = (NK + 3) / 4;
+  static constexpr int NK = NK_, L = L_, NCW = NCW_, STAGES = STAGES_, NB = NB_;
   static constexpr int R = (NK - 1) / 2;
-  static constexpr int ODD = R & 1;
-  static constexpr int SL = ((ODD + L + NK + 4 * KA) + 1) / 2 * 2;  // staged segment length
+  static constexpr int ODD = R & 1;                                  // 16-B aligned copies
+  static constexpr int KS = (NK + 7 + 3) / 4;                        // k-slices per 8 outputs
+  static constexpr int NBLK = L / 8;                                 // 8-output blocks per segment
+  static constexpr int BPW = NBLK / NCW;                             // blocks per consumer warp
+  static constexpr int WIN = 2 * NB + KS - 2;                        // A-fragment register window
+  static constexpr int SLA = ODD + L - 8 + 4 * KS;                   // read by the GEMM
+  static constexpr int SLB = ODD + L + 2 * R;                        // read by the band code
+  static constexpr int SL = ((SLA > SLB ? SLA : SLB) + 1) / 2 * 2;   // staged segment length
   static constexpr int P = s2r_pitch_dev(SL);                        // segment pitch (doubles)
   static constexpr int STAGE = 8 * P;
   static constexpr int TILE = 8 * L;                                 // outputs per tile
   static constexpr int NT = 32 * (NCW + 1);
   static constexpr int SMEM = STAGES * STAGE * 8;
-  static_assert(L % SW == 0, "segment length must be a multiple of nk+1");
+  static_assert(L % 8 == 0 && NBLK % NCW == 0 && BPW % NB == 0, "1D tile geometry");
 };
 
 template <class C>
@@ -586,14 +592,10 @@ __global__ void __launch_bounds__(C::NT, 2) k_tile1d(S2RArgs a) {  // 2 CTAs/SM
     return;
   }
   const int g = lane >> 2, t = lane & 3;
-  double wa[C::NF][C::KA], wb[C::NF][C::KA];
+  double wt[C::KS];  // Toeplitz B fragments: lane (k = t, n = g) of slice q holds w[4q + t - g]
 #pragma unroll
-  for (int f = 0; f < C::NF; ++f)
-#pragma unroll
-    for (int s = 0; s < C::KA; ++s) {
-      wa[f][s] = a.frags[((0 * C::NF + f) * C::KA + s) * 32 + lane];
-      wb[f][s] = a.frags[((1 * C::NF + f) * C::KA + s) * 32 + lane];
-    }
+  for (int q = 0; q < C::KS; ++q) wt[q] = a.frags[q * 32 + lane];
+  const int fb = a.fix_band;
   int it = 0;
   for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
     const int s = it % C::STAGES;
@@ -601,95 +603,81 @@ __global__ void __launch_bounds__(C::NT, 2) k_tile1d(S2RArgs a) {  // 2 CTAs/SM
     const double* seg = smem + s * C::STAGE + g * C::P + C::ODD + t;  // this lane's segment g
     const int64_t tsl = slab_map(a, tile);
     const int64_t t0 = tsl * C::TILE + (int64_t)g * C::L;
-    constexpr int NSTRIP = C::L / C::SW;
-    double res[(NSTRIP + C::NCW - 1) / C::NCW][C::NF][2];
+#pragma unroll 1
+    for (int grp = 0; grp < C::BPW / C::NB; ++grp) {
+      const int b0 = warp * C::BPW + grp * C::NB;
+      double x[C::WIN];
 #pragma unroll
-    for (int q = 0; q < (NSTRIP + C::NCW - 1) / C::NCW; ++q) {
-      const int k = warp + q * C::NCW;
-      if (k < NSTRIP) {
+      for (int i = 0; i < C::WIN; ++i) x[i] = seg[8 * b0 + 4 * i];
+      double acc[C::NB][2];
 #pragma unroll
-        for (int f = 0; f < C::NF; ++f) res[q][f][0] = res[q][f][1] = 0.0;
+      for (int j = 0; j < C::NB; ++j) acc[j][0] = acc[j][1] = 0.0;
 #pragma unroll
-        for (int s2 = 0; s2 < C::KA; ++s2) {
-          const double xa = seg[k * C::SW + 4 * s2];
-          const double xb = seg[k * C::SW + C::NK + 4 * s2];
+      for (int q = 0; q < C::KS; ++q)
 #pragma unroll
-          for (int f = 0; f < C::NF; ++f) {
-            dmma_t(res[q][f][0], res[q][f][1], xa, wa[f][s2]);
-            dmma_t(res[q][f][0], res[q][f][1], xb, wb[f][s2]);
+        for (int j = 0; j < C::NB; ++j) dmma_t(acc[j][0], acc[j][1], x[2 * j + q], wt[q]);
+#pragma unroll
+      for (int j = 0; j < C::NB; ++j) {
+        const int64_t o = t0 + 8 * (b0 + j) + 2 * t;  // outputs o, o+1 of segment g
+        if (fb > 0) {  // band points are written by the band code below
+          const int64_t go = o + a.gorg2;
+          if (o < a.E2 && !(go < fb || go >= a.GE2 - fb)) a.dst.p[o] = acc[j][0];
+          if (o + 1 < a.E2 && !(go + 1 < fb || go + 1 >= a.GE2 - fb)) a.dst.p[o + 1] = acc[j][1];
+          continue;
+        }
+        if (o < a.E2) {
+          double* p = a.dst.p + o;
+          if (o + 1 < a.E2 && ((reinterpret_cast<uintptr_t>(p) & 15) == 0)) {
+            *reinterpret_cast<double2*>(p) = make_double2(acc[j][0], acc[j][1]);
+          } else {
+            p[0] = acc[j][0];
+            if (o + 1 < a.E2) p[1] = acc[j][1];
           }
         }
       }
     }
     // FIXED: the band b = r*Tf at each global end is recomputed by Tf plain steps (reading A1)
-    // by warp 0 from the staged segments, one lane per point, neighbours via shuffles.
-    const int fb = a.fix_band;
+    // by warp 0 from the staged segments, one lane per point, neighbours via shuffles, in
+    // chunks of 32 - 2 r (Tf-1) points (the lanes a chunk's Tf-level cone leaves valid).
     const int64_t tg0 = tsl * C::TILE + a.gorg2;  // global index of the tile's first output
     if (fb > 0 && warp == 0 && (tg0 < fb || tg0 + C::TILE > a.GE2 - fb)) {
-      const int r = a.r, tf = fb / r, D = r * (tf - 1);
+      const int r = a.r, tf = fb / r, D = r * (tf - 1), CH = 32 - 2 * D;
       for (int sg = 0; sg < 8; ++sg) {
         const int64_t s0 = tg0 + (int64_t)sg * C::L;  // global range of segment sg
+        const double* sgm = smem + s * C::STAGE + sg * C::P + C::ODD;  // index = pos - s0 + R
         for (int side = 0; side < 2; ++side) {
           int64_t q0 = side == 0 ? 0 : a.GE2 - fb, q1 = side == 0 ? fb : a.GE2;
           q0 = max(q0, s0);
           q1 = min(q1, min(s0 + (int64_t)C::L, a.GE2));
           q1 = min(q1, a.gorg2 + a.E2);
-          if (q0 >= q1) continue;
-          // lane l <-> global position q0 - D + l; level 0 from the staged segment
-          const int64_t gp = q0 - D + lane;
-          const double* sgm = smem + s * C::STAGE + sg * C::P + C::ODD;  // staged: index = pos - s0 + R
-          const bool hold = gp < r || gp >= a.GE2 - r;
-          const int li = (int)(gp - s0) + C::R;
-          double v = 0.0;
-          if (li >= 0 && li < C::SL) {
-            if (hold) {
-              v = sgm[li];
-            } else {
-              for (int o = -r; o <= r; ++o) v = fma(__ldg(a.wbase + o + r), sgm[li + o], v);
+          for (int64_t qc = q0; qc < q1; qc += CH) {
+            const int64_t gp = qc - D + lane;  // lane <-> global position
+            const bool hold = gp < r || gp >= a.GE2 - r;
+            const int li = (int)(gp - s0) + C::R;
+            double v = 0.0;
+            if (li >= 0 && li < C::SL) {
+              if (hold) {
+                v = sgm[li];
+              } else {
+                for (int o = -r; o <= r; ++o)
+                  if (li + o >= 0 && li + o < C::SL) v = fma(__ldg(a.wbase + o + r), sgm[li + o], v);
+              }
             }
-          }
-          for (int lv = 2; lv <= tf; ++lv) {
-            double nv = 0.0;
-            for (int o = -r; o <= r; ++o) {
-              const double x = __shfl_sync(0xffffffffu, v, (lane + o) & 31);
-              nv = fma(__ldg(a.wbase + o + r), x, nv);
+            for (int lv = 2; lv <= tf; ++lv) {
+              double nv = 0.0;
+              for (int o = -r; o <= r; ++o) {
+                const double xv = __shfl_sync(0xffffffffu, v, (lane + o) & 31);
+                nv = fma(__ldg(a.wbase + o + r), xv, nv);
+              }
+              v = hold ? v : nv;
             }
-            v = hold ? v : nv;
+            if (gp >= qc && gp < min(q1, qc + CH)) a.dst.p[gp - a.gorg2] = v;
           }
-          const int64_t lp = gp - a.gorg2;  // local position
-          if (gp >= q0 && gp < q1 && lane < 32) a.dst.p[lp] = v;
         }
       }
     }
     __syncwarp();
     if (lane == 0) mbar_arrive(&empty[s]);
-#pragma unroll
-    for (int q = 0; q < (NSTRIP + C::NCW - 1) / C::NCW; ++q) {
-      const int k = warp + q * C::NCW;
-      if (k < NSTRIP) {
-#pragma unroll
-        for (int f = 0; f < C::NF; ++f) {
-          const int c = 8 * f + 2 * t;
-          const int64_t o = t0 + (int64_t)k * C::SW + c;
-          if (fb > 0) {  // band points are written by the band code above
-            const int64_t go = o + a.gorg2;
-            if (c < C::SW && o < a.E2 && !(go < fb || go >= a.GE2 - fb)) a.dst.p[o] = res[q][f][0];
-            if (c + 1 < C::SW && o + 1 < a.E2 && !(go + 1 < fb || go + 1 >= a.GE2 - fb))
-              a.dst.p[o + 1] = res[q][f][1];
-            continue;
-          }
-          if (c < C::SW && o < a.E2) {
-            double* p = a.dst.p + o;
-            if (c + 1 < C::SW && o + 1 < a.E2 && ((reinterpret_cast<uintptr_t>(p) & 15) == 0)) {
-              *reinterpret_cast<double2*>(p) = make_double2(res[q][f][0], res[q][f][1]);
-            } else {
-              p[0] = res[q][f][0];
-              if (c + 1 < C::SW && o + 1 < a.E2) p[1] = res[q][f][1];
-            }
-          }
-        }
-      }
-    }
   }
 }
 
@@ -707,22 +695,51 @@ static cudaError_t launch_tile1d_cfg(S2RArgs a, cudaStream_t st) {
   return launch_pdl(a.pdl != 0, k_tile1d<C>, grid, C::NT, C::SMEM, st, a);
 }
 
-// consumer warps / stages per nk as measured on B200 (Heat-1D nk=15: 8 warps, 1D5P nk=13: 4)
+static int tile1d_variant() {
+  static const int v = [] {
+    const char* e = getenv("CSX_TILE1D_VARIANT");
+    return e ? atoi(e) : 0;
+  }();
+  return v;
+}
+
+template <int NK>
+static cudaError_t launch_tile1d_nk(const S2RArgs& a, cudaStream_t st) {
+  if constexpr (NK == 15 || NK == 27 || NK == 29) {  // tuning variants (CSX_TILE1D_VARIANT)
+    switch (tile1d_variant()) {
+      case 1: return launch_tile1d_cfg<Tile1DCfg<NK, 512, 4, 4, 4>>(a, st);
+      case 2: return launch_tile1d_cfg<Tile1DCfg<NK, 256, 4, 6, 2>>(a, st);
+      case 3: return launch_tile1d_cfg<Tile1DCfg<NK, 512, 8, 3, 4>>(a, st);
+      case 4: return launch_tile1d_cfg<Tile1DCfg<NK, 384, 4, 4, 4>>(a, st);
+      case 5: return launch_tile1d_cfg<Tile1DCfg<NK, 128, 4, 8, 4>>(a, st);
+    }
+  }
+  return launch_tile1d_cfg<Tile1DCfg<NK, 256, 4, 6, 4>>(a, st);  // 2 CTAs/SM x 4 DMMA warps
+}
+
 static cudaError_t launch_tile1d(int nk, const S2RArgs& a, cudaStream_t st) {
   switch (nk) {
-    case 3: return launch_tile1d_cfg<Tile1DCfg<3, 256, 4, 6>>(a, st);
-    case 5: return launch_tile1d_cfg<Tile1DCfg<5, 252, 4, 6>>(a, st);
-    case 7: return launch_tile1d_cfg<Tile1DCfg<7, 256, 4, 6>>(a, st);
-    case 9: return launch_tile1d_cfg<Tile1DCfg<9, 250, 4, 6>>(a, st);
-    case 11: return launch_tile1d_cfg<Tile1DCfg<11, 252, 4, 6>>(a, st);
-    case 13: return launch_tile1d_cfg<Tile1DCfg<13, 252, 4, 6>>(a, st);
-    case 15: return launch_tile1d_cfg<Tile1DCfg<15, 256, 8, 5>>(a, st);
+    case 3: return launch_tile1d_nk<3>(a, st);
+    case 5: return launch_tile1d_nk<5>(a, st);
+    case 7: return launch_tile1d_nk<7>(a, st);
+    case 9: return launch_tile1d_nk<9>(a, st);
+    case 11: return launch_tile1d_nk<11>(a, st);
+    case 13: return launch_tile1d_nk<13>(a, st);
+    case 15: return launch_tile1d_nk<15>(a, st);
+    case 17: return launch_tile1d_nk<17>(a, st);
+    case 19: return launch_tile1d_nk<19>(a, st);
+    case 21: return launch_tile1d_nk<21>(a, st);
+    case 23: return launch_tile1d_nk<23>(a, st);
+    case 25: return launch_tile1d_nk<25>(a, st);
+    case 27: return launch_tile1d_nk<27>(a, st);
+    case 29: return launch_tile1d_nk<29>(a, st);
+    case 31: return launch_tile1d_nk<31>(a, st);
   }
   return cudaErrorNotSupported;
 }
 
 bool tile_kernel_exists(int ndim, int nk) {
-  return (ndim == 1 && (nk & 1) && nk >= 3 && nk <= 15) ||
+  return (ndim == 1 && (nk & 1) && nk >= 3 && nk <= 31) ||
          (ndim == 2 && (nk == 3 || nk == 5 || nk == 7)) || (ndim == 3 && nk == 3);
 }
 

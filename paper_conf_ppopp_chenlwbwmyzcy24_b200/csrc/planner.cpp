@@ -262,12 +262,21 @@ csx_status build_pass(const csx_plan_s* p, int tf, Pass* out) {
   // row padded to kc (a multiple of 4) so that every k-slice is 4 consecutive cells of one
   // input row.  Block shape per nk minimises K: nk=3 -> 4x2 (K=24), nk=5 -> 2x4 (K=48),
   // nk=7 -> 4x2 (K=80) versus the paper's 2*ceil(nk^2/4)*4 = 24 / 56 / 104.
-  if (ndim == 1 && P.s2r_ok) {
-    // 1D TC_TILE uses the paper's W_A / W_B fragments unchanged (same GEMM, different M rows)
+  if (ndim == 1) {
+    // 1D TC_TILE: the 8 N columns are 8 consecutive outputs, so the weight operand is the banded
+    // Toeplitz matrix W[k][n] = w[k - n] (0 <= k - n < nk), K = nk + 7 rounded up to 4.
     P.tile_ok = 1;
-    P.tile_frags = P.frags;
-    P.tile_ks = P.ks;
-    P.tile_mma_per_pass = P.mma_per_pass;
+    P.tile_a = 1;
+    P.tile_b = 8;
+    P.tile_ks = (nk + 7 + 3) / 4;
+    P.tile_kc = 4 * P.tile_ks;
+    P.tile_frags.assign((size_t)P.tile_ks * 32, 0.0);
+    for (int s = 0; s < P.tile_ks; ++s)
+      for (int l = 0; l < 32; ++l) {
+        const int k = 4 * s + (l % 4), n = l / 4, j = k - n;
+        P.tile_frags[(size_t)s * 32 + l] = (j >= 0 && j < nk) ? P.wc[j] : 0.0;
+      }
+    P.tile_mma_per_pass = (int64_t)((double)pts / 64.0 * P.tile_ks + 0.5);
   }
   if (ndim >= 2 && nk <= 7) {
     int a = 4, b = 2;
@@ -311,8 +320,10 @@ static int auto_tf(int ndim, int radius) {
 csx_status build_plan(csx_plan_s* p) {
   if (p->tf <= 0) p->tf = auto_tf(p->ndim, p->radius);
   const int nk = 2 * p->radius * p->tf + 1;
-  if (p->ndim == 1 && nk > 15)
-    return fail(CSX_ERR_UNSUPPORTED, "1D: composed window 2*r*Tf+1 must be <= 15");
+  // 1D: TC_S2R (the paper's layout, nf <= 2 N fragments) takes nk <= 15, TC_TILE (Toeplitz
+  // blocks) nk <= 31 — the FIXED band code's 32-lane cone needs 2 r (Tf-1) <= 31.
+  if (p->ndim == 1 && nk > 31)
+    return fail(CSX_ERR_UNSUPPORTED, "1D: composed window 2*r*Tf+1 must be <= 31");
   if (p->ndim == 2 && nk > 7)
     return fail(CSX_ERR_UNSUPPORTED, "2D: composed window 2*r*Tf+1 must be <= 7 (one N fragment)");
   if (p->ndim == 3 && p->tf != 1)

@@ -87,6 +87,32 @@ def test_parity_fusion_depths_1d(csx, tf):
         assert rel(got, oracle.run(u0, w, bc, 23)) <= TOL, (tf, bc)
 
 
+@pytest.mark.parametrize("r,tf", [(1, 1), (1, 3), (1, 7), (1, 8), (1, 11), (1, 15), (2, 3), (2, 5),
+                                  (2, 7), (3, 2), (3, 5)])
+def test_parity_fusion_depths_1d_tile(csx, r, tf):
+    """TC_TILE 1D (Toeplitz blocks, nk = 2 r Tf + 1 up to 31): 3 full tiles of 8 x 256 outputs
+    plus a ragged tail; T = 2 Tf + 3 covers fused passes and a remainder pass."""
+    u0 = synth.grid((3 * 2048 + 777,), seed=60 + r)
+    w = {1: synth.random_weights("heat1d"), 2: synth.random_weights("1d5p")}.get(r)
+    if w is None:
+        w = synth.random_signed_weights(1, r, seed=61)
+    T = 2 * tf + 3
+    for bc in ("fixed", "periodic"):
+        got, info = run_gpu(csx, u0, w, "box", bc, T, engine="tc_tile", fuse_steps=tf)
+        assert info["nk"] == 2 * r * tf + 1
+        assert rel(got, oracle.run(u0, w, bc, T)) <= TOL, (r, tf, bc)
+
+
+def test_1d_deep_fusion_minimum_extent(csx):
+    """Extent = nk exactly (every point is within the band of some face)."""
+    w = synth.random_weights("heat1d")
+    for tf in (8, 15):
+        u0 = synth.grid((2 * tf + 1,), seed=62)
+        for bc in ("fixed", "periodic"):
+            got, _ = run_gpu(csx, u0, w, "box", bc, 2 * tf + 1, engine="tc_tile", fuse_steps=tf)
+            assert rel(got, oracle.run(u0, w, bc, 2 * tf + 1)) <= TOL, (tf, bc)
+
+
 def test_signed_weights_general_radius(csx):
     for ndim, r, ext in [(1, 3, (999,)), (2, 2, (70, 90)), (2, 3, (50, 77))]:
         w = synth.random_signed_weights(ndim, r, seed=9)

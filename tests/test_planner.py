@@ -214,6 +214,27 @@ def test_plan_validation():
     p.close()
 
 
+def test_1d_fusion_limits():
+    """1D: TC_TILE (Toeplitz 8-output blocks, K = nk + 7 rounded up to 4) runs nk <= 31, the
+    paper's stencil2row layout (TC_S2R, nf <= 2) nk <= 15; nk = 33 is refused."""
+    w = synth.physical_weights("heat1d")
+    p = csx.Plan((4096,), w, fuse_steps=15, engine="tc_tile")
+    info = p.info()
+    assert info["nk"] == 31
+    assert info["mma_per_pass"] == 4096 // 64 * 10
+    with pytest.raises(csx.CsxError):
+        p.set_engine("tc_s2r")
+    p.set_engine("auto")
+    p.close()
+    p = csx.Plan((4096,), w, fuse_steps=7, engine="tc_tile")
+    assert p.info()["mma_per_pass"] == 4096 // 64 * 6      # nk = 15: K = 22 -> 24
+    p.set_engine("tc_s2r")                                   # Eq 13: 2 ceil(15/4) nf=2 per 8x16
+    assert p.info()["mma_per_pass"] == 4096 // (8 * 16) * 2 * 4 * 2
+    p.close()
+    with pytest.raises(csx.CsxError):
+        csx.Plan((4096,), w, fuse_steps=16)
+
+
 def test_auto_fusion_depths():
     cases = {"heat1d": 7, "1d5p": 3, "heat2d": 3, "box2d9p": 3, "star2d13p": 1, "box2d49p": 1,
              "heat3d": 1, "box3d27p": 1}
