@@ -24,7 +24,6 @@ import os
 import statistics
 import subprocess
 import sys
-import tempfile
 import time
 
 import numpy as np
@@ -76,26 +75,53 @@ def peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks and throttle reasons sampled every 200 ms during the timed region."""
+    """nvidia-smi clocks and throttle reasons, sampled every 20 ms by a reader thread that stamps
+    each row with the host clock.  The sampler is started (and its first row awaited) before the
+    timed region; mark() brackets the region on the host (the steps are enqueued inside it and it
+    ends after the device synchronize, so it covers the device work).  summary() keeps the rows
+    inside the region plus the one just before and just after it (a region shorter than the
+    sampling period still gets the two samples that bracket it)."""
 
     FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
               "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
               "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
 
-    def __init__(self, gpu_index):
+    def __init__(self, gpu_index, period_ms=20):
         self.gpu = gpu_index
+        self.period = period_ms
         self.proc = None
-        self.tmp = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        self.rows = []  # (host monotonic time, [fields])
+        self.t0 = self.t1 = None
+        self.thread = None
+
+    def _reader(self):
+        for line in self.proc.stdout:
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) >= 9 and parts[1].replace(".", "").isdigit():
+                self.rows.append((time.monotonic(), parts))
 
     def __enter__(self):
+        import threading
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={self.FIELDS}",
-                 "--format=csv,noheader,nounits", "-lms", "200"],
-                stdout=self.tmp, stderr=subprocess.DEVNULL)
+                 "--format=csv,noheader,nounits", "-lms", str(self.period)],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True, bufsize=1)
+            self.thread = threading.Thread(target=self._reader, daemon=True)
+            self.thread.start()
+            deadline = time.monotonic() + 10.0
+            while not self.rows and time.monotonic() < deadline and self.proc.poll() is None:
+                time.sleep(0.01)
         except Exception:
             self.proc = None
         return self
+
+    def mark(self, which):
+        if which == "start":
+            self.t0 = time.monotonic()
+        else:
+            self.t1 = time.monotonic()
+            time.sleep(2.5 * self.period / 1000.0)  # let the row after the region arrive
 
     def __exit__(self, *exc):
         if self.proc:
@@ -104,32 +130,33 @@ class ClockSampler:
                 self.proc.wait(timeout=5)
             except Exception:
                 self.proc.kill()
+        if self.thread:
+            self.thread.join(timeout=2)
 
     def summary(self):
-        self.tmp.flush()
-        rows = []
-        try:
-            with open(self.tmp.name) as f:
-                for line in f:
-                    parts = [x.strip() for x in line.split(",")]
-                    if len(parts) >= 9 and parts[1].replace(".", "").isdigit():
-                        rows.append(parts)
-        except Exception:
-            pass
-        finally:
-            try:
-                os.unlink(self.tmp.name)
-            except Exception:
-                pass
+        rows = list(self.rows)
         if not rows:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
-        sm = [float(r[1]) for r in rows]
-        smax = max(float(r[2]) for r in rows)
-        loaded = [s for s, r in zip(sm, rows) if float(r[3]) > 250.0] or sm
+        t0 = self.t0 if self.t0 is not None else rows[0][0]
+        t1 = self.t1 if self.t1 is not None else rows[-1][0]
+        inside = [r for t, r in rows if t0 <= t <= t1]
+        before = [r for t, r in rows if t < t0][-1:]
+        after = [r for t, r in rows if t > t1][:1]
+        sel = before + inside + after
+        sm = [float(r[1]) for r in sel]
+        smax = max(float(r[2]) for r in sel)
+
+        def power(r):
+            try:
+                return float(r[3])
+            except ValueError:
+                return 0.0
+        loaded = [s for s, r in zip(sm, sel) if power(r) > 250.0] or sm
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({n for r in rows for n, v in zip(names, r[5:9]) if v.lower() == "active"})
+        reasons = sorted({n for r in sel for n, v in zip(names, r[5:9]) if v.lower() == "active"})
         return {"sm_mhz": statistics.median(loaded), "sm_max_mhz": smax, "reasons": reasons,
-                "samples": len(rows)}
+                "samples": len(sel), "samples_inside": len(inside),
+                "timed_region_s": round(t1 - t0, 4), "period_ms": self.period}
 
 
 def algorithmic_mma(ndim, nk, engine, points, tc_planes):
@@ -316,6 +343,7 @@ def main():
            for _ in range(args.steps)]
     with ClockSampler(local) as clk:
         barrier_sync()
+        clk.mark("start")
         for e0, e1 in evs:
             if flush is not None:
                 flush.fill_(1.0)
@@ -323,6 +351,7 @@ def main():
             step()
             e1.record(stream)
         barrier_sync()
+        clk.mark("end")
     ms_total = sum(e0.elapsed_time(e1) for e0, e1 in evs)
     tc_ms, tc_launches, launches = csx.csx_profile_read(plan.handle, reset=True)
     csx.csx_profile_enable(plan.handle, False)

@@ -77,6 +77,11 @@ typedef struct csx_comm_s* csx_comm_t;
 csx_status csx_plan(int ndim, const int64_t* extents, csx_shape shape, int radius,
                     const double* weights, csx_boundary bc, int fuse_steps, csx_plan_t* out);
 
+/* The fusion depth csx_plan picks for fuse_steps = 0 (reading A4), for a plan that
+ * will run on `engine` (AUTO = the depth csx_plan itself uses; TC_S2R 1D keeps the paper's
+ * nk + 1 <= 16).  Returns Tf >= 1, or 0 for ndim / radius / engine out of range.  Host-only. */
+int csx_auto_fuse_steps(int ndim, int radius, csx_engine engine);
+
 /* Select the engine for subsequent runs (default AUTO).  UNSUPPORTED if the engine cannot run
  * this plan's (ndim, radius, Tf). */
 csx_status csx_plan_set_engine(csx_plan_t plan, csx_engine engine);

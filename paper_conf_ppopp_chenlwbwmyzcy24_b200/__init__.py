@@ -58,6 +58,7 @@ def _sig(name, res, args):
 _sig("csx_plan", ctypes.c_int, [ctypes.c_int, _i64p, ctypes.c_int, ctypes.c_int, _dp, ctypes.c_int,
                                 ctypes.c_int, ctypes.POINTER(_vp)])
 _sig("csx_plan_set_engine", ctypes.c_int, [_vp, ctypes.c_int])
+_sig("csx_auto_fuse_steps", ctypes.c_int, [ctypes.c_int, ctypes.c_int, ctypes.c_int])
 _sig("csx_plan_set_s2r_variant", ctypes.c_int, [_vp, ctypes.c_int, ctypes.c_int])
 _sig("csx_run", ctypes.c_int, [_vp, _vp, _vp, ctypes.c_int64, _vp])
 _sig("csx_run_host", ctypes.c_int, [_vp, _dp, _dp, ctypes.c_int64, _vp])
@@ -83,7 +84,7 @@ _sig("csx_profile_read", ctypes.c_int, [_vp, ctypes.POINTER(ctypes.c_double), _i
 
 _sig("csx_halo_schedule", ctypes.c_int, [_vp, ctypes.c_int, ctypes.c_int, _i64p, ctypes.POINTER(ctypes.c_int)])
 
-EXPORTED = ["csx_plan_set_s2r_variant", "csx_halo_schedule", "csx_profile_enable", "csx_profile_read", "csx_plan", "csx_plan_set_engine", "csx_run", "csx_run_host", "csx_comm_create",
+EXPORTED = ["csx_auto_fuse_steps", "csx_plan_set_s2r_variant", "csx_halo_schedule", "csx_profile_enable", "csx_profile_read", "csx_plan", "csx_plan_set_engine", "csx_run", "csx_run_host", "csx_comm_create",
             "csx_comm_destroy", "csx_nccl_unique_id", "csx_shard_rows", "csx_run_sharded",
             "csx_plan_destroy", "csx_status_string", "csx_last_error", "csx_plan_info",
             "csx_compose_weights", "csx_weight_matrices", "csx_stencil2row_index",
@@ -284,6 +285,9 @@ class Plan:
             raise ValueError("weights must have one axis per grid axis")
         self.radius = (w.shape[0] - 1) // 2
         self.n = int(np.prod(self.extents))
+        if fuse_steps == 0 and engine != "auto":
+            # the automatic depth for the requested engine (TC_S2R 1D keeps nk + 1 <= 16)
+            fuse_steps = int(_lib.csx_auto_fuse_steps(self.ndim, self.radius, ENGINES[engine]))
         self._h = csx_plan(self.ndim, self.extents, CSX_SHAPE_BOX if shape == "box" else CSX_SHAPE_STAR,
                            self.radius, w, CSX_BC_FIXED if bc == "fixed" else CSX_BC_PERIODIC,
                            fuse_steps)

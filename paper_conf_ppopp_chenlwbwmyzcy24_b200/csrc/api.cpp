@@ -341,6 +341,12 @@ csx_status csx_plan(int ndim, const int64_t* extents, csx_shape shape, int radiu
   return CSX_OK;
 }
 
+int csx_auto_fuse_steps(int ndim, int radius, csx_engine engine) {
+  if (ndim < 1 || ndim > 3 || radius < 1 || radius > 3) return 0;
+  if (engine < CSX_ENGINE_AUTO || engine > CSX_ENGINE_DIRECT) return 0;
+  return csx::auto_tf(ndim, radius, engine);
+}
+
 csx_status csx_plan_set_s2r_variant(csx_plan_t p, int padding, int dirty_bits) {
   if (!p) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL plan");
   // padding = 2: breakdown variant II (padding + dirty bits, tessellation on CUDA cores)
@@ -572,7 +578,7 @@ csx_status run_local(csx_plan_s* p, const double* d_in, double* d_out, int64_t T
     const int tfp = i < nmain ? p->tf : rem;
     const bool last = i == npass - 1;
     PassCtx c;
-    c.src = CView{b[cur].p, b[cur].s0, b[cur].s1};
+    c.src = CView{b[cur].p, b[cur].s0, b[cur].s1, pd.O[0], pd.O[1], pd.O[2], pd.A[0]};
     c.dst = last ? out : b[cur ^ 1];
     for (int a = 0; a < 3; ++a) { c.E[a] = p->E[a]; c.gorg[a] = 0; }
     csx_status s = run_pass(p, p->passes[tfp - 1], c, st);

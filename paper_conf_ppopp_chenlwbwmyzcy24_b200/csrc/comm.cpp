@@ -236,7 +236,7 @@ csx_status csx_run_sharded(csx_plan_t p, csx_comm_t c, const double* d_in, doubl
     const int tfp = i < nmain ? p->tf : rem;
     const bool last = i == npass - 1;
     PassCtx pc;
-    pc.src = CView{b[cur].p, b[cur].s0, b[cur].s1};
+    pc.src = CView{b[cur].p, b[cur].s0, b[cur].s1, pd.O[0], pd.O[1], pd.O[2], pd.A[0]};
     pc.dst = last ? out : b[cur ^ 1];
     for (int a = 0; a < 3; ++a) { pc.E[a] = El[a]; pc.gorg[a] = 0; }
     pc.gorg[a0] = lo;

@@ -126,6 +126,7 @@ struct csx_plan_s {
 namespace csx {
 // planner.cpp
 csx_status build_plan(csx_plan_s* p);
+int auto_tf(int ndim, int radius, int engine);  // automatic fusion depth (reading A4)
 csx_status build_pass(const csx_plan_s* p, int tf, Pass* out);
 void layout_padded(const csx_plan_s* p, const int64_t* E, Padded* pd);
 }  // namespace csx

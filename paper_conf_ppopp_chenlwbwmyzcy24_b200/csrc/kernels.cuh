@@ -13,6 +13,10 @@ struct View {
 struct CView {
   const double* p;
   int64_t s0, s1;
+  // allocation geometry of a padded grid (for TMA tensor maps): interior origin inside the
+  // allocation and the number of allocated planes (rows = s0 / s1, row pitch = s1).
+  // n0 == 0: unknown (kernels fall back to per-row bulk copies).
+  int64_t o0 = 0, o1 = 0, o2 = 0, n0 = 0;
 };
 
 struct S2RArgs {
@@ -37,6 +41,8 @@ struct S2RArgs {
   int fix_band = 0;
   int pdl = 1;                    // TC_TILE: launch with programmatic dependent launch
   int hold_frame = 0;             // write held (frame) values from the staged tile (Tf = 1)
+  int use_tma = 0;                // TC_TILE 2D/3D: stage tiles with one TMA tensor copy
+  int64_t tma_x0 = 0, tma_y0 = 0, tma_z0 = 0;  // interior origin in tensor-map coordinates
   int r = 0;
   const double* wbase = nullptr;  // base weights (2r+1)^2
   int64_t gorg0 = 0, gorg1 = 0, gorg2 = 0;  // local origin in global coordinates

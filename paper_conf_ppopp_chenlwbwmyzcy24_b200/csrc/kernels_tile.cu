@@ -13,6 +13,8 @@
 //   * the input tile is staged by cp.async.bulk (TMA bulk copies, one per row) into a
 //     double-buffered smem ring with mbarrier completion, so the next tile streams in while the
 //     DMMA pipe works on the current one (persistent CTAs, 2 per SM).
+#include <cuda.h>
+#include <cudaTypedefs.h>
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -61,6 +63,65 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
           "r"(smem_u32(dst)),
       "l"(src), "r"(bytes), "r"(smem_u32(bar))
       : "memory");
+}
+
+// TMA tensor copy of one box {x, y, z} (elements, innermost first) of the padded source grid
+// into smem, completing on `bar` (expect_tx set by the caller).  One instruction per staged
+// tile / plane instead of one bulk copy per row (the per-row loop was the 3D producer's
+// bottleneck: ~66 serialised UBLKCP per plane).
+__device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, uint64_t* bar, int x,
+                                            int y, int z) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%2, %3, %4}], [%5];\n" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(z), "r"(smem_u32(bar))
+      : "memory");
+}
+
+__device__ __forceinline__ void tma_prefetch_desc(const CUtensorMap* map) {
+  asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(map)) : "memory");
+}
+
+// 128-B aligned base of the dynamic smem ring (TMA tensor destinations need 128 B alignment)
+// (offset arithmetic on the __shared__ array itself, so the compiler keeps LDS addressing)
+__device__ __forceinline__ double* ring_base(double* raw) {
+  return raw + ((128u - (smem_u32(raw) & 127u)) & 127u) / 8u;
+}
+
+// Host: a rank-3 tensor map over the whole allocation of a padded grid (FP64, no swizzle, box
+// {bx, by, 1}); fills the interior origin in tensor-map coordinates.  Returns false (caller
+// falls back to per-row bulk copies) if the geometry is unknown or the driver entry point is
+// missing.
+static bool make_tmap(S2RArgs& a, int bx, int by, CUtensorMap* map) {
+  static PFN_cuTensorMapEncodeTiled_v12000 encode = [] {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess) {
+      cudaGetLastError();
+      return (PFN_cuTensorMapEncodeTiled_v12000) nullptr;
+    }
+    return reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+  }();
+  const char* e = getenv("CSX_TMA");
+  if (e && e[0] == '0') return false;
+  const CView& v = a.src;
+  if (!encode || v.n0 <= 0 || v.s1 <= 0 || v.s0 % v.s1 != 0) return false;
+  const double* base = v.p - (v.o0 * v.s0 + v.o1 * v.s1 + v.o2);
+  if ((reinterpret_cast<uintptr_t>(base) & 15) != 0 || (v.s1 * 8) % 16 != 0) return false;
+  cuuint64_t dims[3] = {(cuuint64_t)v.s1, (cuuint64_t)(v.s0 / v.s1), (cuuint64_t)v.n0};
+  cuuint64_t strides[2] = {(cuuint64_t)v.s1 * 8, (cuuint64_t)v.s0 * 8};
+  cuuint32_t box[3] = {(cuuint32_t)bx, (cuuint32_t)by, 1};
+  cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = encode(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, const_cast<double*>(base), dims,
+                      strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                      CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return false;
+  a.use_tma = 1;
+  a.tma_x0 = v.o2;
+  a.tma_y0 = v.o1;
+  a.tma_z0 = v.o0;
+  return true;
 }
 
 // Programmatic dependent launch (sm_90+): the kernels below are launched with programmatic
@@ -159,18 +220,28 @@ struct TileCfg {
   static constexpr int BN = WN * WC;                // CTA output cols
   static constexpr int RR = BM + NK - 1;            // staged input rows
   static constexpr int TP = ((ODD + BN + KC - B) + 1) / 2 * 2;  // staged row length (even)
-  static constexpr int STAGE = RR * TP;             // doubles per stage
+  static constexpr int STAGE = RR * TP;             // doubles staged per tile
+  static constexpr int STAGE_A = (STAGE + 15) / 16 * 16;  // ring slot (128-B aligned)
   static constexpr int NCW = WM * WN;               // consumer (DMMA) warps
   static constexpr int NT = 32 * (NCW + 1);         // + one producer warp
-  static constexpr int SMEM = STAGES * STAGE * 8;
+  static constexpr int SMEM = STAGES * STAGE_A * 8 + 128;
+  static_assert(TP <= 256 && RR <= 256, "TMA box dimensions");
 };
 
 template <class C>
-__device__ __forceinline__ void issue_tile(const S2RArgs& a, int64_t tile, double* stage,
-                                           uint64_t* bar, int lane) {
+__device__ __forceinline__ void issue_tile(const S2RArgs& a, const CUtensorMap* tmap, int64_t tile,
+                                           double* stage, uint64_t* bar, int lane) {
   const int64_t tyl = tile / a.tiles_x;
   const int tx = (int)(tile - tyl * a.tiles_x);
   const int ty = (int)slab_map(a, tyl);
+  if (a.use_tma) {
+    if (lane == 0) {
+      mbar_expect_tx(bar, (uint32_t)(C::STAGE * 8));
+      tma_load_3d(stage, tmap, bar, (int)(a.tma_x0 + tx * C::BN - C::R - C::ODD),
+                  (int)(a.tma_y0 + (int64_t)ty * C::BM - C::R), (int)a.tma_z0);
+    }
+    return;
+  }
   const double* src = a.src.p + (int64_t)(ty * C::BM - C::R) * a.src.s1 + (tx * C::BN - C::R - C::ODD);
   if (lane == 0) mbar_expect_tx(bar, (uint32_t)(C::STAGE * 8));
   __syncwarp();
@@ -189,8 +260,10 @@ __device__ __forceinline__ bool tile_is_edge(const S2RArgs& a, int ty, int tx) {
 // Warp-specialised persistent kernel: warp NCW is the producer (bulk copies of the input tile
 // into a STAGES-deep smem ring, full/empty mbarriers); warps 0..NCW-1 run the DMMA GEMM.
 template <class C>
-__global__ void __launch_bounds__(C::NT, C::MINB) k_tile2d(S2RArgs a) {
-  extern __shared__ __align__(128) double smem[];
+__global__ void __launch_bounds__(C::NT, C::MINB)
+    k_tile2d(S2RArgs a, const __grid_constant__ CUtensorMap tmap) {
+  extern __shared__ __align__(128) double smem_raw[];
+  double* smem = ring_base(smem_raw);
   __shared__ __align__(8) uint64_t full[C::STAGES], empty[C::STAGES];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   if (tid == 0) {
@@ -205,11 +278,12 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_tile2d(S2RArgs a) {
   if (warp == C::NCW) {
     // ---------------- producer ----------------
     int it = 0;
+    if (a.use_tma && lane == 0) tma_prefetch_desc(&tmap);
     for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
       const int s = it % C::STAGES;
       const int n = it / C::STAGES;
       if (n > 0) mbar_wait(&empty[s], (n - 1) & 1);
-      issue_tile<C>(a, tile, smem + s * C::STAGE, &full[s], lane);
+      issue_tile<C>(a, &tmap, tile, smem + s * C::STAGE_A, &full[s], lane);
     }
     return;
   }
@@ -228,7 +302,7 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_tile2d(S2RArgs a) {
     const int64_t tyl = tile / a.tiles_x;
     const int tx = (int)(tile - tyl * a.tiles_x);
     const int ty = (int)slab_map(a, tyl);
-    const double* base = smem + s * C::STAGE + (wm * C::A * C::G) * C::TP + wn * C::WC + C::ODD +
+    const double* base = smem + s * C::STAGE_A + (wm * C::A * C::G) * C::TP + wn * C::WC + C::ODD +
                          C::B * g + t;
     double acc[C::CG][C::G][2];
 #pragma unroll
@@ -308,7 +382,7 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_tile2d(S2RArgs a) {
             double v = acc[cg][j][e];
             if (rowband || gc < a.fix_band || gc >= a.GE2 - a.fix_band) {
               if (!a.hold_frame) continue;
-              v = smem[s * C::STAGE + (int)(row - (int64_t)ty * C::BM + C::R) * C::TP +
+              v = smem[s * C::STAGE_A + (int)(row - (int64_t)ty * C::BM + C::R) * C::TP +
                        (int)(c - (int64_t)tx * C::BN) + C::R + C::ODD];
             }
             a.dst.p[row * a.dst.s1 + c] = v;
@@ -368,15 +442,26 @@ struct Tile3DCfg {
   static constexpr int RR = BM + NK - 1;
   static constexpr int TP = ((ODD + BN + KC - B) + 1) / 2 * 2;
   static constexpr int STAGE = RR * TP;
+  static constexpr int STAGE_A = (STAGE + 15) / 16 * 16;  // ring slot (128-B aligned)
+  static constexpr bool TMA_ONLY = true;  // no per-row bulk-copy fallback (launcher requires the map)
   static constexpr int NCW = WM * WN;
   static constexpr int NT = 32 * (NCW + 1);
-  static constexpr int SMEM = STAGES * STAGE * 8;
+  static constexpr int SMEM = STAGES * STAGE_A * 8 + 128;
   static_assert(STAGES >= NK + 1, "plane ring must hold NK planes plus one in flight");
+  static_assert(TP <= 256 && RR <= 256, "TMA box dimensions");
 };
 
 template <class C>
-__device__ __forceinline__ void issue_plane(const S2RArgs& a, int ty, int tx, int64_t zi, double* stage,
-                                            uint64_t* bar, int lane) {
+__device__ __forceinline__ void issue_plane(const S2RArgs& a, const CUtensorMap* tmap, int ty, int tx,
+                                            int64_t zi, double* stage, uint64_t* bar, int lane) {
+  if (C::TMA_ONLY || a.use_tma) {
+    if (lane == 0) {
+      mbar_expect_tx(bar, (uint32_t)(C::STAGE * 8));
+      tma_load_3d(stage, tmap, bar, (int)(a.tma_x0 + tx * C::BN - C::R - C::ODD),
+                  (int)(a.tma_y0 + (int64_t)ty * C::BM - C::R), (int)(a.tma_z0 + zi));
+    }
+    return;
+  }
   const double* src = a.src.p + zi * a.src.s0 + (int64_t)(ty * C::BM - C::R) * a.src.s1 +
                       (tx * C::BN - C::R - C::ODD);
   if (lane == 0) mbar_expect_tx(bar, (uint32_t)(C::STAGE * 8));
@@ -386,8 +471,10 @@ __device__ __forceinline__ void issue_plane(const S2RArgs& a, int ty, int tx, in
 }
 
 template <class C>
-__global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2)) k_tile3d(S2RArgs a, int tc_mask) {
-  extern __shared__ __align__(128) double smem[];
+__global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
+    k_tile3d(S2RArgs a, int tc_mask, const __grid_constant__ CUtensorMap tmap) {
+  extern __shared__ __align__(128) double smem_raw[];
+  double* smem = ring_base(smem_raw);
   __shared__ __align__(8) uint64_t full[C::STAGES], empty[C::STAGES];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   if (tid == 0) {
@@ -401,6 +488,7 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2)) k_tile3d(S2RArgs 
   pdl_begin();  // PDL: let the next pass launch; wait for the previous pass's writes
   const int64_t ncol = (int64_t)a.tiles_x * a.tiles_y;
   if (warp == C::NCW) {  // producer: planes of every work item, in consumption order
+    if (a.use_tma && lane == 0) tma_prefetch_desc(&tmap);
     int64_t q = 0;
     for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
       const int64_t zcl = item / ncol, tile = item - zcl * ncol;
@@ -411,7 +499,7 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2)) k_tile3d(S2RArgs 
         const int s = (int)(q % C::STAGES);
         const int64_t n = q / C::STAGES;
         if (n > 0) mbar_wait(&empty[s], (uint32_t)((n - 1) & 1));
-        issue_plane<C>(a, ty, tx, zi, smem + s * C::STAGE, &full[s], lane);
+        issue_plane<C>(a, &tmap, ty, tx, zi, smem + s * C::STAGE_A, &full[s], lane);
       }
     }
     return;
@@ -450,7 +538,7 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2)) k_tile3d(S2RArgs 
 #pragma unroll
       for (int dz = 0; dz < C::NK; ++dz) {
         const int64_t qp = q0 + (zo - z0) + dz;  // plane zo - R + dz
-        const double* stg = smem + (qp % C::STAGES) * C::STAGE;
+        const double* stg = smem + (qp % C::STAGES) * C::STAGE_A;
         if (tc_mask & (1 << dz)) {
           const double* base = stg + (wm * C::A * C::G) * C::TP + wn * 8 * C::B + C::ODD + C::B * g + t;
 #pragma unroll
@@ -485,7 +573,7 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2)) k_tile3d(S2RArgs 
                         (plane_frame || (int64_t)ty * C::BM + a.gorg1 < C::R ||
                          (int64_t)(ty + 1) * C::BM + a.gorg1 > a.GE1 - C::R ||
                          (int64_t)tx * C::BN + a.gorg2 < C::R || (int64_t)(tx + 1) * C::BN + a.gorg2 > a.GE2 - C::R);
-      const double* cstg = smem + ((q0 + (zo - z0) + C::R) % C::STAGES) * C::STAGE;
+      const double* cstg = smem + ((q0 + (zo - z0) + C::R) % C::STAGES) * C::STAGE_A;
       double* plane = a.dst.p + zo * a.dst.s0;
 #pragma unroll
       for (int j = 0; j < C::G; ++j) {
@@ -705,13 +793,15 @@ static int tile1d_variant() {
 
 template <int NK>
 static cudaError_t launch_tile1d_nk(const S2RArgs& a, cudaStream_t st) {
-  if constexpr (NK == 15 || NK == 27 || NK == 29) {  // tuning variants (CSX_TILE1D_VARIANT)
+  if constexpr (NK == 15 || NK == 19 || NK == 21 || NK == 23) {  // tuning variants (CSX_TILE1D_VARIANT)
     switch (tile1d_variant()) {
       case 1: return launch_tile1d_cfg<Tile1DCfg<NK, 512, 4, 4, 4>>(a, st);
       case 2: return launch_tile1d_cfg<Tile1DCfg<NK, 256, 4, 6, 2>>(a, st);
       case 3: return launch_tile1d_cfg<Tile1DCfg<NK, 512, 8, 3, 4>>(a, st);
       case 4: return launch_tile1d_cfg<Tile1DCfg<NK, 384, 4, 4, 4>>(a, st);
       case 5: return launch_tile1d_cfg<Tile1DCfg<NK, 128, 4, 8, 4>>(a, st);
+      case 6: return launch_tile1d_cfg<Tile1DCfg<NK, 256, 8, 4, 4>>(a, st);
+      case 7: return launch_tile1d_cfg<Tile1DCfg<NK, 256, 4, 6, 8>>(a, st);
     }
   }
   return launch_tile1d_cfg<Tile1DCfg<NK, 256, 4, 6, 4>>(a, st);  // 2 CTAs/SM x 4 DMMA warps
@@ -750,6 +840,8 @@ static cudaError_t launch_tile_cfg(S2RArgs a, cudaStream_t st) {
   a.tiles_y = (int)((a.E1 + C::BM - 1) / C::BM);
   a.ntiles = (int64_t)a.tiles_x * set_ranges(a, a.tiles_y, C::BM, a.E1, C::R);
   if (a.ntiles == 0) return cudaSuccess;
+  CUtensorMap tmap;
+  if (!make_tmap(a, C::TP, C::RR, &tmap)) a.use_tma = 0;
   cudaError_t e = cudaFuncSetAttribute(k_tile2d<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
   if (e != cudaSuccess) return e;
   int occ = 0;
@@ -757,7 +849,7 @@ static cudaError_t launch_tile_cfg(S2RArgs a, cudaStream_t st) {
   if (e != cudaSuccess) return e;
   int64_t grid = cap_grid(a, (int64_t)(occ < 1 ? 1 : occ) * num_sms());
   if (grid > a.ntiles) grid = a.ntiles;
-  return launch_pdl(a.pdl != 0, k_tile2d<C>, grid, C::NT, C::SMEM, st, a);
+  return launch_pdl(a.pdl != 0, k_tile2d<C>, grid, C::NT, C::SMEM, st, a, tmap);
 }
 
 template <class C>
@@ -766,6 +858,8 @@ static cudaError_t launch_tile3d_cfg(S2RArgs a, int tc_mask, cudaStream_t st) {
   a.tiles_y = (int)((a.E1 + C::BM - 1) / C::BM);
   a.ntiles = (int64_t)a.tiles_x * a.tiles_y * set_ranges(a, (a.E0 + C::ZCH - 1) / C::ZCH, C::ZCH, a.E0, C::R);
   if (a.ntiles == 0) return cudaSuccess;
+  CUtensorMap tmap;
+  if (!make_tmap(a, C::TP, C::RR, &tmap)) return cudaErrorNotSupported;  // 3D stages by TMA only
   cudaError_t e = cudaFuncSetAttribute(k_tile3d<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
   if (e != cudaSuccess) return e;
   int occ = 0;
@@ -773,7 +867,7 @@ static cudaError_t launch_tile3d_cfg(S2RArgs a, int tc_mask, cudaStream_t st) {
   if (e != cudaSuccess) return e;
   int64_t grid = cap_grid(a, (int64_t)(occ < 1 ? 1 : occ) * num_sms());
   if (grid > a.ntiles) grid = a.ntiles;
-  return launch_pdl(a.pdl != 0, k_tile3d<C>, grid, C::NT, C::SMEM, st, a, tc_mask);
+  return launch_pdl(a.pdl != 0, k_tile3d<C>, grid, C::NT, C::SMEM, st, a, tc_mask, tmap);
 }
 
 cudaError_t launch_tile(int ndim, int nk, const S2RArgs& a, cudaStream_t st) {

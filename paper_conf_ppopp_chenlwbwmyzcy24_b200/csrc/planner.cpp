@@ -308,17 +308,23 @@ csx_status build_pass(const csx_plan_s* p, int tf, Pass* out) {
   return CSX_OK;
 }
 
-static int auto_tf(int ndim, int radius) {
-  // 2D r=1 -> 3 (the paper's Box-2D9P choice, P.1478-1480);
-  // r >= 2 in 2D and all 3D -> 1 (one N fragment, lowest DMMA count per point-step on B200);
-  // 1D -> the deepest fusion that keeps nk + 1 <= 16 (HBM-bound regime).
-  if (ndim == 1) return radius == 1 ? 7 : (radius == 2 ? 3 : 2);
+int auto_tf(int ndim, int radius, int engine) {
+  // DESIGN.md "Fusion depth" (reading A4): 2D r=1 -> 3 (the paper's Box-2D9P choice,
+  // P.1478-1480); r >= 2 in 2D and all 3D -> 1 (one N fragment, lowest DMMA count per
+  // point-step on B200).  1D is HBM-bound, so deeper fusion pays until the DMMA work of the
+  // Toeplitz blocks (K = nk + 7) meets the HBM time: TC_TILE takes nk ~ 19..23 (r=1 -> 11,
+  // r=2 -> 5, r=3 -> 3; measured sweep in DESIGN.md §12); TC_S2R's paper layout keeps
+  // nk + 1 <= 16 (two N fragments): r=1 -> 7, r=2 -> 3, r=3 -> 2.
+  if (ndim == 1) {
+    if (engine == CSX_ENGINE_TC_S2R) return radius == 1 ? 7 : (radius == 2 ? 3 : 2);
+    return radius == 1 ? 11 : (radius == 2 ? 5 : 3);
+  }
   if (ndim == 2) return radius == 1 ? 3 : 1;
   return 1;
 }
 
 csx_status build_plan(csx_plan_s* p) {
-  if (p->tf <= 0) p->tf = auto_tf(p->ndim, p->radius);
+  if (p->tf <= 0) p->tf = auto_tf(p->ndim, p->radius, CSX_ENGINE_AUTO);
   const int nk = 2 * p->radius * p->tf + 1;
   // 1D: TC_S2R (the paper's layout, nf <= 2 N fragments) takes nk <= 15, TC_TILE (Toeplitz
   // blocks) nk <= 31 — the FIXED band code's 32-lane cone needs 2 r (Tf-1) <= 31.

@@ -236,7 +236,7 @@ def test_1d_fusion_limits():
 
 
 def test_auto_fusion_depths():
-    cases = {"heat1d": 7, "1d5p": 3, "heat2d": 3, "box2d9p": 3, "star2d13p": 1, "box2d49p": 1,
+    cases = {"heat1d": 11, "1d5p": 5, "heat2d": 3, "box2d9p": 3, "star2d13p": 1, "box2d49p": 1,
              "heat3d": 1, "box3d27p": 1}
     for name, tf in cases.items():
         s = synth.SHAPES[name]
@@ -244,6 +244,13 @@ def test_auto_fusion_depths():
         p = csx.Plan(ext, synth.physical_weights(name), shape=s.kind)
         assert p.info()["fuse_steps"] == tf, name
         p.close()
+    # an explicit engine gets its own automatic depth: the paper's 1D layout keeps nk + 1 <= 16
+    for name, tf in {"heat1d": 7, "1d5p": 3}.items():
+        p = csx.Plan((4096,), synth.physical_weights(name), engine="tc_s2r")
+        assert p.info()["fuse_steps"] == tf and p.info()["engine_name"] == "tc_s2r", name
+        p.close()
+    assert csx._lib.csx_auto_fuse_steps(1, 3, csx.ENGINES["tc_tile"]) == 3
+    assert csx._lib.csx_auto_fuse_steps(4, 1, 0) == 0
 
 
 def test_shard_rows_partition():
