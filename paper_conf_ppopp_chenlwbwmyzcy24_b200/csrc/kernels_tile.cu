@@ -88,6 +88,19 @@ __device__ __forceinline__ double* ring_base(double* raw) {
   return raw + ((128u - (smem_u32(raw) & 127u)) & 127u) / 8u;
 }
 
+static CUtensorMapL2promotion tma_promotion() {
+  static const int v = [] {
+    const char* e = getenv("CSX_TMA_PROMO");
+    return e ? atoi(e) : 0;
+  }();
+  switch (v) {
+    case 64: return CU_TENSOR_MAP_L2_PROMOTION_L2_64B;
+    case 128: return CU_TENSOR_MAP_L2_PROMOTION_L2_128B;
+    case 256: return CU_TENSOR_MAP_L2_PROMOTION_L2_256B;
+  }
+  return CU_TENSOR_MAP_L2_PROMOTION_NONE;
+}
+
 // Host: a rank-3 tensor map over the whole allocation of a padded grid (FP64, no swizzle, box
 // {bx, by, 1}); fills the interior origin in tensor-map coordinates.  Returns false (caller
 // falls back to per-row bulk copies) if the geometry is unknown or the driver entry point is
@@ -115,7 +128,7 @@ static bool make_tmap(S2RArgs& a, int bx, int by, CUtensorMap* map) {
   cuuint32_t estr[3] = {1, 1, 1};
   CUresult r = encode(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, const_cast<double*>(base), dims,
                       strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                      CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                      tma_promotion(), CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return false;
   a.use_tma = 1;
   a.tma_x0 = v.o2;
@@ -429,21 +442,21 @@ static int tile_variant() {
 // DMMA warps compute output plane zo from the NK staged planes zo-R .. zo+R (every tensor-core z
 // offset is a K-slice group of the same GEMM; single-tap z offsets — the star arms, reading A9 —
 // are DFMAs on the same staged planes), then release plane zo-R, which no later output needs.
-template <int NK_, int G_, int WM_, int WN_, int STAGES_, int ZCH_>
+template <int NK_, int G_, int WM_, int WN_, int STAGES_, int ZCH_, int CG_ = 1>
 struct Tile3DCfg {
   static constexpr int NK = NK_, A = 4, B = 2, KC = 4 * ((2 + NK - 1 + 3) / 4), G = G_, WM = WM_,
-                       WN = WN_, STAGES = STAGES_, ZCH = ZCH_;
+                       WN = WN_, STAGES = STAGES_, ZCH = ZCH_, CG = CG_;
   static constexpr int R = (NK - 1) / 2;
-  static constexpr int ODD = R & 1;
+  static constexpr int ODD = R & 1;  // staged col = region col + ODD (16-B aligned rows)
   static constexpr int KR = A + NK - 1;
   static constexpr int KS = KR * KC / 4;
   static constexpr int BM = WM * A * G;
-  static constexpr int BN = WN * 8 * B;
+  static constexpr int WC = CG * 8 * B;             // output cols per warp (CG column groups)
+  static constexpr int BN = WN * WC;
   static constexpr int RR = BM + NK - 1;
   static constexpr int TP = ((ODD + BN + KC - B) + 1) / 2 * 2;
   static constexpr int STAGE = RR * TP;
   static constexpr int STAGE_A = (STAGE + 15) / 16 * 16;  // ring slot (128-B aligned)
-  static constexpr bool TMA_ONLY = true;  // no per-row bulk-copy fallback (launcher requires the map)
   static constexpr int NCW = WM * WN;
   static constexpr int NT = 32 * (NCW + 1);
   static constexpr int SMEM = STAGES * STAGE_A * 8 + 128;
@@ -454,21 +467,14 @@ struct Tile3DCfg {
 template <class C>
 __device__ __forceinline__ void issue_plane(const S2RArgs& a, const CUtensorMap* tmap, int ty, int tx,
                                             int64_t zi, double* stage, uint64_t* bar, int lane) {
-  if (C::TMA_ONLY || a.use_tma) {
-    if (lane == 0) {
-      mbar_expect_tx(bar, (uint32_t)(C::STAGE * 8));
-      tma_load_3d(stage, tmap, bar, (int)(a.tma_x0 + tx * C::BN - C::R - C::ODD),
-                  (int)(a.tma_y0 + (int64_t)ty * C::BM - C::R), (int)(a.tma_z0 + zi));
-    }
-    return;
+  if (lane == 0) {
+    mbar_expect_tx(bar, (uint32_t)(C::STAGE * 8));
+    tma_load_3d(stage, tmap, bar, (int)(a.tma_x0 + tx * C::BN - C::R - C::ODD),
+                (int)(a.tma_y0 + (int64_t)ty * C::BM - C::R), (int)(a.tma_z0 + zi));
   }
-  const double* src = a.src.p + zi * a.src.s0 + (int64_t)(ty * C::BM - C::R) * a.src.s1 +
-                      (tx * C::BN - C::R - C::ODD);
-  if (lane == 0) mbar_expect_tx(bar, (uint32_t)(C::STAGE * 8));
-  __syncwarp();
-  for (int r = lane; r < C::RR; r += 32)
-    bulk_g2s(stage + r * C::TP, src + (int64_t)r * a.src.s1, (uint32_t)(C::TP * 8), bar);
 }
+
+__device__ __forceinline__ int ring_next(int s, int n) { return s + 1 == n ? 0 : s + 1; }
 
 template <class C>
 __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
@@ -486,20 +492,22 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
   }
   __syncthreads();
   pdl_begin();  // PDL: let the next pass launch; wait for the previous pass's writes
-  const int64_t ncol = (int64_t)a.tiles_x * a.tiles_y;
+  const int ncol = a.tiles_x * a.tiles_y;
   if (warp == C::NCW) {  // producer: planes of every work item, in consumption order
-    if (a.use_tma && lane == 0) tma_prefetch_desc(&tmap);
-    int64_t q = 0;
+    if (lane == 0) tma_prefetch_desc(&tmap);
+    int s = 0, round = 0;  // ring slot and how many times the ring has been filled
     for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
-      const int64_t zcl = item / ncol, tile = item - zcl * ncol;
+      const int zcl = (int)(item / ncol), tile = (int)(item - (int64_t)zcl * ncol);
       const int64_t zc = slab_map(a, zcl);
-      const int ty = (int)(tile / a.tiles_x), tx = (int)(tile - (int64_t)ty * a.tiles_x);
+      const int ty = tile / a.tiles_x, tx = tile - ty * a.tiles_x;
       const int64_t z0 = zc * C::ZCH, z1 = min(a.E0, z0 + C::ZCH);
-      for (int64_t zi = z0 - C::R; zi < z1 + C::R; ++zi, ++q) {
-        const int s = (int)(q % C::STAGES);
-        const int64_t n = q / C::STAGES;
-        if (n > 0) mbar_wait(&empty[s], (uint32_t)((n - 1) & 1));
+      for (int64_t zi = z0 - C::R; zi < z1 + C::R; ++zi) {
+        if (round > 0) mbar_wait(&empty[s], (uint32_t)((round - 1) & 1));
         issue_plane<C>(a, &tmap, ty, tx, zi, smem + s * C::STAGE_A, &full[s], lane);
+        if (++s == C::STAGES) {
+          s = 0;
+          ++round;
+        }
       }
     }
     return;
@@ -511,111 +519,144 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
 #pragma unroll
   for (int p = 0; p < C::NK; ++p) {
 #pragma unroll
-    for (int s = 0; s < C::KS; ++s) wf[p][s] = a.frags[(p * C::KS + s) * 32 + lane];
+    for (int k = 0; k < C::KS; ++k) wf[p][k] = a.frags[(p * C::KS + k) * 32 + lane];
     wz[p] = a.wc[(p * C::NK + C::R) * C::NK + C::R];
   }
   const int alpha = (2 * t) / C::B, beta = (2 * t) % C::B;
   const bool any_cuda = tc_mask != (1 << C::NK) - 1;
-  int64_t q0 = 0;  // plane sequence number of the current item's first plane
+  const bool aligned = a.dst_aligned != 0;
+  // ring position / phase of the next plane this warp consumes (planes are consumed in issue
+  // order, so slot = sequence number mod STAGES and phase = (sequence / STAGES) & 1)
+  int cs = 0;
+  uint32_t cph = 0;
+  // lane-invariant offsets inside a staged plane
+  const int lane_off = (wm * C::A * C::G) * C::TP + wn * C::WC + C::ODD + C::B * g + t;
+  const int frame_off = (wm * C::A * C::G + alpha + C::R) * C::TP + wn * C::WC + C::B * g + beta +
+                        C::R + C::ODD;
   for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
-    const int64_t zcl = item / ncol, tile = item - zcl * ncol;
+    const int zcl = (int)(item / ncol), tile = (int)(item - (int64_t)zcl * ncol);
     const int64_t zc = slab_map(a, zcl);
-    const int ty = (int)(tile / a.tiles_x), tx = (int)(tile - (int64_t)ty * a.tiles_x);
+    const int ty = tile / a.tiles_x, tx = tile - ty * a.tiles_x;
     const int64_t z0 = zc * C::ZCH, z1 = min(a.E0, z0 + C::ZCH);
-    const int64_t col = (int64_t)tx * C::BN + wn * 8 * C::B + C::B * g + beta;
+    const int64_t col0 = (int64_t)tx * C::BN + wn * C::WC + C::B * g + beta;
     const int64_t row0 = (int64_t)ty * C::BM + wm * C::A * C::G + alpha;
-    // planes z0-R .. z0+R-1 are needed before the first output plane
-    for (int k = 0; k < 2 * C::R; ++k) {
-      const int64_t qq = q0 + k;
-      mbar_wait(&full[qq % C::STAGES], (uint32_t)((qq / C::STAGES) & 1));
-    }
-    for (int64_t zo = z0; zo < z1; ++zo) {
-      const int64_t qn = q0 + (zo - z0) + 2 * C::R;  // newest plane zo + R
-      mbar_wait(&full[qn % C::STAGES], (uint32_t)((qn / C::STAGES) & 1));
-      double acc[C::G][2];
+    const bool full_tile = aligned && (int64_t)(ty + 1) * C::BM <= a.E1 && (int64_t)(tx + 1) * C::BN <= a.E2;
+    const bool tile_edge = a.hold_frame &&
+                           ((int64_t)ty * C::BM + a.gorg1 < C::R || (int64_t)(ty + 1) * C::BM + a.gorg1 > a.GE1 - C::R ||
+                            (int64_t)tx * C::BN + a.gorg2 < C::R || (int64_t)(tx + 1) * C::BN + a.gorg2 > a.GE2 - C::R);
+    // slots of the NK planes zo-R .. zo+R of the current output plane
+    int slot[C::NK];
+    uint32_t sph[C::NK];
+    slot[0] = cs;
+    sph[0] = cph;
 #pragma unroll
-      for (int j = 0; j < C::G; ++j) acc[j][0] = acc[j][1] = 0.0;
+    for (int k = 1; k < C::NK; ++k) {
+      slot[k] = ring_next(slot[k - 1], C::STAGES);
+      sph[k] = slot[k] == 0 ? sph[k - 1] ^ 1 : sph[k - 1];
+    }
+#pragma unroll
+    for (int k = 0; k < C::NK - 1; ++k) mbar_wait(&full[slot[k]], sph[k]);
+    for (int64_t zo = z0; zo < z1; ++zo) {
+      mbar_wait(&full[slot[C::NK - 1]], sph[C::NK - 1]);  // newest plane zo + R
+      double acc[C::CG][C::G][2];
+#pragma unroll
+      for (int cg = 0; cg < C::CG; ++cg)
+#pragma unroll
+        for (int j = 0; j < C::G; ++j) acc[cg][j][0] = acc[cg][j][1] = 0.0;
 #pragma unroll
       for (int dz = 0; dz < C::NK; ++dz) {
-        const int64_t qp = q0 + (zo - z0) + dz;  // plane zo - R + dz
-        const double* stg = smem + (qp % C::STAGES) * C::STAGE_A;
+        const double* stg = smem + slot[dz] * C::STAGE_A;
         if (tc_mask & (1 << dz)) {
-          const double* base = stg + (wm * C::A * C::G) * C::TP + wn * 8 * C::B + C::ODD + C::B * g + t;
+          const double* base = stg + lane_off;
 #pragma unroll
           for (int ra = 0; ra < C::A * C::G + C::NK - 1; ++ra) {
-            double f[C::KC / 4];
+            double f[C::CG][C::KC / 4];
 #pragma unroll
-            for (int h = 0; h < C::KC / 4; ++h) f[h] = base[ra * C::TP + 4 * h];
+            for (int cg = 0; cg < C::CG; ++cg)
+#pragma unroll
+              for (int h = 0; h < C::KC / 4; ++h) f[cg][h] = base[ra * C::TP + cg * 8 * C::B + 4 * h];
 #pragma unroll
             for (int h = 0; h < C::KC / 4; ++h)
 #pragma unroll
               for (int j = 0; j < C::G; ++j) {
                 const int rho = ra - C::A * j;
                 if (rho >= 0 && rho < C::KR)
-                  dmma_t(acc[j][0], acc[j][1], f[h], wf[dz][rho * (C::KC / 4) + h]);
+#pragma unroll
+                  for (int cg = 0; cg < C::CG; ++cg)
+                    dmma_t(acc[cg][j][0], acc[cg][j][1], f[cg][h], wf[dz][rho * (C::KC / 4) + h]);
               }
           }
         } else if (any_cuda && wz[dz] != 0.0) {
 #pragma unroll
-          for (int j = 0; j < C::G; ++j) {
-            const int lr = wm * C::A * C::G + C::A * j + alpha + C::R;
-            const int lc = wn * 8 * C::B + C::B * g + beta + C::R + C::ODD;
-            const double2 v = *reinterpret_cast<const double2*>(stg + lr * C::TP + lc);
-            acc[j][0] = fma(wz[dz], v.x, acc[j][0]);
-            acc[j][1] = fma(wz[dz], v.y, acc[j][1]);
-          }
+          for (int cg = 0; cg < C::CG; ++cg)
+#pragma unroll
+            for (int j = 0; j < C::G; ++j) {
+              const double2 v = *reinterpret_cast<const double2*>(stg + frame_off + C::A * j * C::TP + cg * 8 * C::B);
+              acc[cg][j][0] = fma(wz[dz], v.x, acc[cg][j][0]);
+              acc[cg][j][1] = fma(wz[dz], v.y, acc[cg][j][1]);
+            }
         }
       }
       // FIXED frame (held points) of this output plane: the staged plane zo (dz = R) holds them
       const int64_t gzo = zo + a.gorg0;
       const bool plane_frame = a.hold_frame && (gzo < C::R || gzo >= a.GE0 - C::R);
-      const bool edge = a.hold_frame &&
-                        (plane_frame || (int64_t)ty * C::BM + a.gorg1 < C::R ||
-                         (int64_t)(ty + 1) * C::BM + a.gorg1 > a.GE1 - C::R ||
-                         (int64_t)tx * C::BN + a.gorg2 < C::R || (int64_t)(tx + 1) * C::BN + a.gorg2 > a.GE2 - C::R);
-      const double* cstg = smem + ((q0 + (zo - z0) + C::R) % C::STAGES) * C::STAGE_A;
       double* plane = a.dst.p + zo * a.dst.s0;
+      if (full_tile && !tile_edge && !plane_frame) {  // interior: unguarded 16-B stores
+        double* p0 = plane + row0 * a.dst.s1 + col0;
 #pragma unroll
-      for (int j = 0; j < C::G; ++j) {
-        const int64_t row = row0 + C::A * j;
-        if (row < a.E1 && col < a.E2) {
-          double* p = plane + row * a.dst.s1 + col;
-          if (!edge) {
-            if (col + 1 < a.E2 && ((reinterpret_cast<uintptr_t>(p) & 15) == 0)) {
-              *reinterpret_cast<double2*>(p) = make_double2(acc[j][0], acc[j][1]);
-            } else {
-              p[0] = acc[j][0];
-              if (col + 1 < a.E2) p[1] = acc[j][1];
-            }
-          } else {
+        for (int cg = 0; cg < C::CG; ++cg)
+#pragma unroll
+          for (int j = 0; j < C::G; ++j)
+            *reinterpret_cast<double2*>(p0 + (int64_t)(C::A * j) * a.dst.s1 + cg * 8 * C::B) =
+                make_double2(acc[cg][j][0], acc[cg][j][1]);
+      } else {
+        const double* cstg = smem + slot[C::R] * C::STAGE_A;
+        const bool edge = tile_edge || plane_frame;
+#pragma unroll
+        for (int cg = 0; cg < C::CG; ++cg)
+#pragma unroll
+          for (int j = 0; j < C::G; ++j) {
+            const int64_t row = row0 + C::A * j, col = col0 + cg * 8 * C::B;
+            if (row >= a.E1 || col >= a.E2) continue;
+            double* p = plane + row * a.dst.s1 + col;
             const int64_t grow = row + a.gorg1;
             const bool rf = plane_frame || grow < C::R || grow >= a.GE1 - C::R;
 #pragma unroll
             for (int e = 0; e < 2; ++e) {
               const int64_t c = col + e, gc = c + a.gorg2;
               if (c >= a.E2) continue;
-              double v = acc[j][e];
-              if (rf || gc < C::R || gc >= a.GE2 - C::R)
-                v = cstg[(int)(row - (int64_t)ty * C::BM + C::R) * C::TP + (int)(c - (int64_t)tx * C::BN) + C::R + C::ODD];
+              double v = acc[cg][j][e];
+              if (edge && (rf || gc < C::R || gc >= a.GE2 - C::R))
+                v = cstg[frame_off + C::A * j * C::TP + cg * 8 * C::B + e];
               p[e] = v;
             }
           }
-        }
       }
       __syncwarp();
-      if (lane == 0) mbar_arrive(&empty[(q0 + (zo - z0)) % C::STAGES]);  // plane zo-R is done
+      if (lane == 0) mbar_arrive(&empty[slot[0]]);  // plane zo-R is done
+      // advance the window by one plane
+#pragma unroll
+      for (int k = 0; k < C::NK - 1; ++k) {
+        slot[k] = slot[k + 1];
+        sph[k] = sph[k + 1];
+      }
+      slot[C::NK - 1] = ring_next(slot[C::NK - 2], C::STAGES);
+      sph[C::NK - 1] = slot[C::NK - 1] == 0 ? sph[C::NK - 2] ^ 1 : sph[C::NK - 2];
     }
     // release the last 2R planes of the item (not released by an output plane)
     __syncwarp();
     if (lane == 0)
-      for (int k = 0; k < 2 * C::R; ++k) mbar_arrive(&empty[(q0 + (z1 - z0) + k) % C::STAGES]);
-    q0 += (z1 - z0) + 2 * C::R;
+#pragma unroll
+      for (int k = 0; k < C::NK - 1; ++k) mbar_arrive(&empty[slot[k]]);
+    cs = slot[C::NK - 1];
+    cph = sph[C::NK - 1];
   }
 }
 
-using Tile3D3 = Tile3DCfg<3, 8, 2, 2, 5, 32>;  // CTA 64 x 32 outputs, 4 DMMA warps, 5-plane ring, 32 planes per item
-using Tile3D3b = Tile3DCfg<3, 4, 4, 4, 4, 32>;  // CTA 64 x 64 outputs, 16 DMMA warps, 1 CTA/SM
-using Tile3D3c = Tile3DCfg<3, 8, 2, 4, 6, 32>;  // CTA 64 x 64 outputs, 8 DMMA warps, 6-plane ring
+using Tile3D3 = Tile3DCfg<3, 8, 2, 2, 5, 32>;      // CTA 64 x 32 outputs, 4 DMMA warps, 5-plane ring, 32 planes per item
+using Tile3D3b = Tile3DCfg<3, 4, 4, 1, 5, 32, 2>;  // CTA 64 x 32, 4 warps of 4 block rows x 2 column groups
+using Tile3D3c = Tile3DCfg<3, 8, 2, 4, 6, 32>;     // CTA 64 x 64 outputs, 8 DMMA warps, 6-plane ring
+using Tile3D3d = Tile3DCfg<3, 2, 8, 1, 5, 32, 2>;  // CTA 64 x 32, 8 warps of 2 block rows x 2 column groups
 
 
 // ------------------------------------------------------------------------------------------
@@ -854,6 +895,8 @@ static cudaError_t launch_tile_cfg(S2RArgs a, cudaStream_t st) {
 
 template <class C>
 static cudaError_t launch_tile3d_cfg(S2RArgs a, int tc_mask, cudaStream_t st) {
+  a.dst_aligned = ((reinterpret_cast<uintptr_t>(a.dst.p) & 15) == 0) && (a.dst.s1 % 2 == 0) &&
+                  (a.dst.s0 % 2 == 0);
   a.tiles_x = (int)((a.E2 + C::BN - 1) / C::BN);
   a.tiles_y = (int)((a.E1 + C::BM - 1) / C::BM);
   a.ntiles = (int64_t)a.tiles_x * a.tiles_y * set_ranges(a, (a.E0 + C::ZCH - 1) / C::ZCH, C::ZCH, a.E0, C::R);
@@ -877,6 +920,12 @@ cudaError_t launch_tile(int ndim, int nk, const S2RArgs& a, cudaStream_t st) {
       const char* e = getenv("CSX_TILE3D_VARIANT");
       if (e && e[0] == '1') return launch_tile3d_cfg<Tile3D3b>(a, a.tc_mask, st);
       if (e && e[0] == '2') return launch_tile3d_cfg<Tile3D3c>(a, a.tc_mask, st);
+      if (e && e[0] == '3') return launch_tile3d_cfg<Tile3D3d>(a, a.tc_mask, st);
+      if (e && e[0] == '0') return launch_tile3d_cfg<Tile3D3>(a, a.tc_mask, st);
+      // default: star shapes (one TC plane, HBM-bound) take the 64 x 64 tile with 8 DMMA warps
+      // (less halo per plane); box shapes (DMMA-bound) the 64 x 32 tile at 2 CTAs / SM
+      // (measured)
+      if (__builtin_popcount((unsigned)a.tc_mask) <= 1) return launch_tile3d_cfg<Tile3D3c>(a, a.tc_mask, st);
       return launch_tile3d_cfg<Tile3D3>(a, a.tc_mask, st);
     }
     return cudaErrorNotSupported;
