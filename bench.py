@@ -252,7 +252,7 @@ def main():
     ap.add_argument("--T", type=int, default=None, help="custom workload: base time steps")
     ap.add_argument("--bc", default=None, choices=["fixed", "periodic"])
     ap.add_argument("--fuse", type=int, default=None, help="override the fusion depth Tf")
-    ap.add_argument("--s2r-variant", default="V", choices=["II", "III", "IV", "V"],
+    ap.add_argument("--s2r-variant", default="V", choices=["I", "II", "III", "IV", "V"],
                     help="TC_S2R breakdown variant (Fig 6): II CUDA-core tessellation, III no padding/"
                          "no dirty bits, IV padding, V full")
     ap.add_argument("--no-e2e", action="store_true")
@@ -295,7 +295,9 @@ def main():
     w = synth.physical_weights(shape)
     gext = (ext[0] * world,) + tuple(ext[1:])  # weak scaling: ext per GPU
     plan = csx.Plan(gext, w, shape=s.kind, bc=bc, fuse_steps=tf, engine=args.engine)
-    if args.s2r_variant == "II":
+    if args.s2r_variant == "I":
+        plan.set_s2r_variant(padding=3, dirty_bits=True)
+    elif args.s2r_variant == "II":
         plan.set_s2r_variant(padding=2, dirty_bits=True)
     elif args.s2r_variant != "V":
         plan.set_s2r_variant(padding=args.s2r_variant == "IV", dirty_bits=False)

@@ -90,7 +90,11 @@ csx_status csx_plan_set_engine(csx_plan_t plan, csx_engine engine);
  * stencil2row pitch nk*rr (Fig 5's conflicting 266) instead of the conflict-free one (268);
  * dirty_bits = 0 replaces the dirty-bits padding by conditional stores in the LUT copy loop.
  * (1, 1) is the paper's full design (the default); (0, 0) = variant III, (1, 0) = IV;
- * padding = 2 selects variant II (same tiles, the tessellation GEMM on CUDA cores / DFMA). */
+ * padding = 2 selects variant II (same tiles, the tessellation GEMM on CUDA cores / DFMA);
+ * padding = 3 selects variant I (explicit stencil2row: A and B materialised in global memory
+ * by an Eq 5/6 div/mod transform kernel, then the tessellation on CUDA cores reading them back;
+ * the plan allocates ~2 nk/(nk+1) x the grid of scratch at the first run).
+ * INVALID_ARGUMENT for padding outside 0..3; UNSUPPORTED for non-default variants in 1D/3D. */
 csx_status csx_plan_set_s2r_variant(csx_plan_t plan, int padding, int dirty_bits);
 
 /* Advance d_in by `timesteps` base steps into d_out (both prod(extents) doubles, device,

@@ -141,9 +141,10 @@ def csx_plan_set_engine(plan, engine: int):
 
 
 def csx_plan_set_s2r_variant(plan, padding=True, dirty_bits: bool = True):
-    """padding: True/False, or 2 for breakdown variant II (CUDA-core tessellation)."""
-    _check(_lib.csx_plan_set_s2r_variant(plan, 2 if padding == 2 else int(bool(padding)),
-                                         int(bool(dirty_bits))), "csx_plan_set_s2r_variant")
+    """padding: True/False, 2 for breakdown variant II (CUDA-core tessellation) or 3 for
+    variant I (explicit stencil2row in global memory)."""
+    pad = padding if (padding in (2, 3) and not isinstance(padding, bool)) else int(bool(padding))
+    _check(_lib.csx_plan_set_s2r_variant(plan, pad, int(bool(dirty_bits))), "csx_plan_set_s2r_variant")
 
 
 def csx_run(plan, d_in, d_out, timesteps: int, n: int, stream=None):

@@ -208,7 +208,20 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
           for (int dz = 0; dz < ps.nk; ++dz) tc_mask |= ps.plane_is_tc[dz] << dz;
         }
       }
-      e = launch_s2r(p->ndim, ps.nk, ps.nf, a, tc_mask, st);
+      if (p->s2r_explicit && p->ndim == 2) {
+        const int64_t need = s2r_explicit_elems(ps.nk, c.E[1], c.E[2]);
+        if (need > p->s2r_elems) {
+          cudaFree(p->d_s2r);
+          p->d_s2r = nullptr;
+          p->s2r_elems = 0;
+          CSX_CUDA(cudaMalloc(&p->d_s2r, (size_t)need * sizeof(double)), "cudaMalloc(stencil2row)");
+          p->s2r_elems = need;
+        }
+        e = launch_s2r_explicit(ps.nk, c.src, c.dst, c.E, ps.d_wc, p->d_s2r, st);
+        p->n_launches += 1;  // two kernels: transform + tessellation
+      } else {
+        e = launch_s2r(p->ndim, ps.nk, ps.nf, a, tc_mask, st);
+      }
     }
     if (e != cudaSuccess) return cuda_fail(e, "TC pass launch");
     if (prof) CSX_CUDA(cudaEventRecord(ev1, st), "cudaEventRecord");
@@ -349,9 +362,13 @@ int csx_auto_fuse_steps(int ndim, int radius, csx_engine engine) {
 
 csx_status csx_plan_set_s2r_variant(csx_plan_t p, int padding, int dirty_bits) {
   if (!p) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL plan");
-  // padding = 2: breakdown variant II (padding + dirty bits, tessellation on CUDA cores)
+  // padding = 2: breakdown variant II (padding + dirty bits, tessellation on CUDA cores);
+  // padding = 3: breakdown variant I (explicit stencil2row in HBM, CUDA-core tessellation)
+  if (padding < 0 || padding > 3) return fail(CSX_ERR_INVALID_ARGUMENT, "padding must be 0..3");
+  if (padding == 3 && p->ndim != 2) return fail(CSX_ERR_UNSUPPORTED, "breakdown variants are 2D only");
   p->s2r_fma = padding == 2;
-  if (p->s2r_fma) { padding = 1; dirty_bits = 1; }
+  p->s2r_explicit = padding == 3;
+  if (p->s2r_fma || p->s2r_explicit) { padding = 1; dirty_bits = 1; }
   if (p->ndim != 2 && !(padding && dirty_bits))
     return fail(CSX_ERR_UNSUPPORTED, "breakdown variants are 2D only");
   p->s2r_pad = padding != 0;
@@ -483,6 +500,7 @@ csx_status csx_plan_destroy(csx_plan_t p) {
     cudaFree(p->d_dense);
     cudaFree(p->d_sbuf[0]);
     cudaFree(p->d_sbuf[1]);
+    cudaFree(p->d_s2r);
 
     cudaSetDevice(cur);
   }

@@ -98,6 +98,9 @@ struct csx_plan_s {
   bool s2r_pad = true;             // TC_S2R 2D: conflict-free pitch (Fig 5)
   bool s2r_dirty = true;           // TC_S2R 2D: dirty-bits padding instead of branches
   bool s2r_fma = false;            // TC_S2R 2D: breakdown II, tessellation on CUDA cores
+  bool s2r_explicit = false;       // TC_S2R 2D: breakdown I, explicit stencil2row in HBM
+  double* d_s2r = nullptr;         // breakdown I: global stencil2row A|B scratch
+  int64_t s2r_elems = 0;
   csx_engine engine = CSX_ENGINE_TC_S2R;
   std::vector<csx::Pass> passes;   // index tf' - 1, for tf' = 1..tf
   // device state (allocated at the first run)

@@ -86,6 +86,11 @@ cudaError_t launch_band(int ndim, int r, int tf, CView src, View dst, const int6
 cudaError_t launch_frame_copy(CView src, View dst, const int64_t* E, const int64_t* gorg,
                               const int64_t* GE, const int* real, int r, cudaStream_t st);
 int s2r_smem_bytes(int ndim, int nk, int nf);
+// Breakdown variant I (kernels_s2r_explicit.cu): explicit stencil2row A/B in global memory
+// (scratch of s2r_explicit_elems doubles) + dual tessellation on CUDA cores.  2D only.
+int64_t s2r_explicit_elems(int nk, int64_t E1, int64_t E2);
+cudaError_t launch_s2r_explicit(int nk, CView src, View dst, const int64_t* E, const double* wc,
+                                double* scratch, cudaStream_t st);
 int num_sms();
 
 }  // namespace csx

@@ -4,7 +4,7 @@ OUT=gpurun_out/breakdown.jsonl
 : > $OUT
 CFG=${1:-box2d9p_10240}
 python bench.py --config $CFG --engine direct --steps 3 --warmup 3 --no-cpu-baseline --no-e2e --no-comparator >> $OUT
-for v in II III IV V; do
+for v in I II III IV V; do
   python bench.py --config $CFG --engine tc_s2r --s2r-variant $v --steps 3 --warmup 3 --no-cpu-baseline --no-e2e --no-comparator >> $OUT
 done
 python bench.py --config $CFG --engine tc_tile --steps 3 --warmup 3 --no-cpu-baseline --no-e2e --no-comparator >> $OUT

@@ -228,21 +228,23 @@ def test_direct_comparator_2d_all_radii(csx):
             assert rel(got, oracle.run(u0, w, bc, 9)) <= TOL, (r, tf, bc)
 
 
-@pytest.mark.parametrize("pad,dirty", [(0, 0), (1, 0), (0, 1), (1, 1), (2, 1)])
-def test_s2r_breakdown_variants(csx, pad, dirty):
-    """Fig 6 breakdown variants of TC_S2R (no padding / no dirty bits) compute the same result."""
-    for name in ("box2d9p", "heat2d", "box2d49p"):
+@pytest.mark.parametrize("pad,dirty", [(0, 0), (1, 0), (0, 1), (1, 1), (2, 1), (3, 1)])
+@pytest.mark.parametrize("bc", ["fixed", "periodic"])
+def test_s2r_breakdown_variants(csx, pad, dirty, bc):
+    """Fig 6 breakdown variants of TC_S2R (I explicit stencil2row, II CUDA-core tessellation, no
+    padding / no dirty bits) compute the same result, over ragged extents and a remainder pass."""
+    for name in ("box2d9p", "heat2d", "box2d49p", "box2d25p"):
         s = synth.SHAPES[name]
         w = synth.random_weights(name)
         u0 = synth.grid((99, 140), seed=51)
-        p = csx.Plan(u0.shape, w, shape=s.kind, bc="fixed", engine="tc_s2r")
-        p.set_s2r_variant(2 if pad == 2 else bool(pad), bool(dirty))
+        p = csx.Plan(u0.shape, w, shape=s.kind, bc=bc, engine="tc_s2r")
+        p.set_s2r_variant(pad if pad in (2, 3) else bool(pad), bool(dirty))
         d_in = torch.from_numpy(u0).cuda()
         d_out = torch.empty_like(d_in)
         p.run(d_in, d_out, 7)
         torch.cuda.synchronize()
         p.close()
-        assert rel(d_out.cpu().numpy(), oracle.run(u0, w, "fixed", 7)) <= TOL, (name, pad, dirty)
+        assert rel(d_out.cpu().numpy(), oracle.run(u0, w, bc, 7)) <= TOL, (name, pad, dirty)
 
 
 @pytest.mark.parametrize("name,ext,T", [("box2d9p", (400, 130), 10), ("heat1d", (30000,), 23),

@@ -274,7 +274,13 @@ def test_s2r_variant_tables():
     assert len(np.unique(live)) == len(live) == 8 * 7 * 38
     p.set_s2r_variant(padding=True, dirty_bits=True)
     assert p.info()["s2r_pitch"] == 268
+    p.set_s2r_variant(padding=3)  # breakdown I: explicit stencil2row (same LUT/pitch tables)
+    assert p.info()["s2r_pitch"] == 268
+    assert csx._lib.csx_plan_set_s2r_variant(p.handle, 4, 1) == csx.CSX_ERR_INVALID_ARGUMENT
     p.close()
+    q = csx.Plan((4096,), synth.physical_weights("heat1d"), engine="tc_s2r")
+    assert csx._lib.csx_plan_set_s2r_variant(q.handle, 3, 1) == csx.CSX_ERR_UNSUPPORTED
+    q.close()
 
 
 def test_run_argument_validation_without_gpu():
