@@ -255,6 +255,8 @@ def main():
     ap.add_argument("--s2r-variant", default="V", choices=["I", "II", "III", "IV", "V"],
                     help="TC_S2R breakdown variant (Fig 6): II CUDA-core tessellation, III no padding/"
                          "no dirty bits, IV padding, V full")
+    ap.add_argument("--exchange", default="peer", choices=["peer", "nccl"],
+                    help="N > 1 halo exchange: SM peer stores over NVLink (default) or NCCL send/recv")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-comparator", action="store_true")
@@ -286,9 +288,17 @@ def main():
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world != args.gpus:
         raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
-    torch.cuda.set_device(local)
+    # CSX_BENCH_SHARE_GPU=1: every rank on cuda:0 (exercises the N > 1 path on a 1-GPU box;
+    # time-sliced, so not a scaling number)
+    share = os.environ.get("CSX_BENCH_SHARE_GPU") == "1"
+    device = 0 if share else local
+    torch.cuda.set_device(device)
+    red_dev = "cpu" if share else "cuda"  # gloo (shared-GPU test mode) reduces on CPU
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if share:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
 
     shape, ext, T, bc, tf = CONFIGS[args.config]
     s = synth.SHAPES[shape]
@@ -305,10 +315,31 @@ def main():
     engine = info["engine_name"]
     stream = torch.cuda.current_stream()
     comm = None
+    exchange = None
     if world > 1:
-        uid = [csx.csx_nccl_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(uid, src=0)
-        comm = csx.csx_comm_create(uid[0], rank, world)
+        exchange = args.exchange
+        if exchange == "peer":
+            # halo exchange by SM peer stores over NVLink (CUDA IPC), epoch flags in peer memory;
+            # if the IPC mapping is refused, every rank switches to the NCCL exchange
+            err = None
+            try:
+                plan.peer_setup(rank, world)
+            except Exception as e:  # noqa: BLE001  (reported in the JSON line)
+                err = repr(e)
+            errs = [None] * world
+            dist.all_gather_object(errs, err)
+            if any(errs):
+                msg = next(e for e in errs if e)
+                if share:  # shared-GPU test mode: NCCL cannot put two ranks on one GPU
+                    raise SystemExit(f"peer setup failed: {msg}")
+                print(f"[bench] peer setup failed, using NCCL: {msg}", file=sys.stderr)
+                exchange = "nccl (peer setup failed: " + msg[:120] + ")"
+                plan.close()
+                plan = csx.Plan(gext, w, shape=s.kind, bc=bc, fuse_steps=tf, engine=args.engine)
+        if not exchange.startswith("peer"):
+            uid = [csx.csx_nccl_unique_id() if rank == 0 else None]
+            dist.broadcast_object_list(uid, src=0)
+            comm = csx.csx_comm_create(uid[0], rank, world)
         lo, hi = plan.shard_rows(rank, world)
         u0 = synth.grid(gext, rows=(lo, hi))
     else:
@@ -318,8 +349,10 @@ def main():
     n_local = u0.size
 
     def step():
-        if comm is None:
+        if world == 1:
             plan.run(d_in, d_out, T, stream)
+        elif comm is None:
+            plan.run_sharded_peer(d_in, d_out, T, n_local, stream)
         else:
             plan.run_sharded(comm, d_in, d_out, T, n_local, stream)
 
@@ -343,7 +376,7 @@ def main():
         flush = torch.empty(32 << 20, dtype=torch.float64, device="cuda")
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
            for _ in range(args.steps)]
-    with ClockSampler(local) as clk:
+    with ClockSampler(device) as clk:
         barrier_sync()
         clk.mark("start")
         for e0, e1 in evs:
@@ -358,7 +391,7 @@ def main():
     tc_ms, tc_launches, launches = csx.csx_profile_read(plan.handle, reset=True)
     csx.csx_profile_enable(plan.handle, False)
     if world > 1:
-        t = torch.tensor([ms_total], device="cuda", dtype=torch.float64)
+        t = torch.tensor([ms_total], device=red_dev, dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms_total = float(t.item())
     ms_step = ms_total / args.steps
@@ -409,6 +442,7 @@ def main():
                        "fuse_steps": tfm, "nk": nk, "engine": engine,
                        "s2r_variant": args.s2r_variant if engine == "tc_s2r" else None,
                        "parallelism": f"slab{world}" if world > 1 else "single",
+                       "exchange": exchange,
                        "l2": ("L2 flushed (256 MB write) between timed steps" if flush is not None
                               else f"inputs larger than L2 ({u0.nbytes >> 20} MB per grid vs 126 MB); no flush")},
             "gpu_launches": int(launches), "roofline": roof}
@@ -466,12 +500,13 @@ def main():
             h_out.copy_(d_out, non_blocking=True)
             e1.record(stream)
             barrier_sync()
-            ems = torch.tensor([e0.elapsed_time(e1)], device="cuda", dtype=torch.float64)
+            ems = torch.tensor([e0.elapsed_time(e1)], device=red_dev, dtype=torch.float64)
             dist.all_reduce(ems, op=dist.ReduceOp.MAX)
             ems = float(ems.item())
             line["e2e"] = {"value": T * points / (ems * 1e-3) / 1e9, "unit": UNIT,
                            "h2d_bytes_per_step": int(u0.nbytes), "d2h_bytes_per_step": int(u0.nbytes),
-                           "api": "torch pinned copies + csx_run_sharded", "ms_per_step": ems}
+                           "api": "torch pinned copies + csx_run_sharded" + ("_peer" if comm is None else ""),
+                           "ms_per_step": ems}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_oracle_sample(shape, gext, T, bc, w)
     if rank == 0:

@@ -136,6 +136,30 @@ csx_status csx_halo_schedule(const csx_plan_t plan, int rank, int nranks, int64_
 csx_status csx_run_sharded(csx_plan_t plan, csx_comm_t comm, const double* d_in_local,
                            double* d_out_local, int64_t timesteps, void* stream);
 
+/* ----- Slab halo exchange over NVLink peer memory (no NCCL on the data path) -----------
+ * The same slab decomposition and results as csx_run_sharded, but after every pass the
+ * boundary slab rows are copied by SM peer stores straight into the neighbours' ghost rows
+ * (CUDA IPC mappings of their plan-owned slab buffers over NVLink / NVSwitch), and readiness is
+ * signalled by 64-bit epoch flags in peer memory (fence + st.release.sys / ld.acquire.sys).
+ * Bootstrap, once per plan, collectively:
+ *   1. every rank calls csx_peer_export(plan, rank, nranks, desc) — allocates this rank's slab
+ *      buffers and flag block (fixed from then on) and writes CSX_PEER_DESC_BYTES of IPC handles
+ *      and geometry into desc;
+ *   2. the caller all-gathers the descriptors in rank order (e.g. torch.distributed
+ *      all_gather_object) and every rank calls csx_peer_connect(plan, descs) with the
+ *      nranks * CSX_PEER_DESC_BYTES array — it maps the up / down neighbours (a rank that is its
+ *      own neighbour, 1-rank PERIODIC, uses its own buffers).
+ * Then csx_run_sharded_peer(plan, d_in_local, d_out_local, T, stream) on every rank with equal T.
+ * Errors: INVALID_ARGUMENT (bad rank, export twice, connect before export, descriptors from a
+ * different plan or out of rank order), UNSUPPORTED (fewer than r*Tf rows per rank), CUDA (IPC
+ * failures).  Ranks spin on device flags: every rank must make progress (one process per GPU,
+ * or time-sliced processes sharing a GPU in tests). */
+#define CSX_PEER_DESC_BYTES 512
+csx_status csx_peer_export(csx_plan_t plan, int rank, int nranks, void* desc);
+csx_status csx_peer_connect(csx_plan_t plan, const void* descs);
+csx_status csx_run_sharded_peer(csx_plan_t plan, const double* d_in_local, double* d_out_local,
+                                int64_t timesteps, void* stream);
+
 csx_status csx_plan_destroy(csx_plan_t plan);
 
 const char* csx_status_string(csx_status s);

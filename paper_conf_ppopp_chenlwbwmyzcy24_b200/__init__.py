@@ -67,6 +67,9 @@ _sig("csx_comm_destroy", ctypes.c_int, [_vp])
 _sig("csx_nccl_unique_id", ctypes.c_int, [ctypes.c_char_p])
 _sig("csx_shard_rows", ctypes.c_int, [_vp, ctypes.c_int, ctypes.c_int, _i64p, _i64p])
 _sig("csx_run_sharded", ctypes.c_int, [_vp, _vp, _vp, _vp, ctypes.c_int64, _vp])
+_sig("csx_peer_export", ctypes.c_int, [_vp, ctypes.c_int, ctypes.c_int, ctypes.c_char_p])
+_sig("csx_peer_connect", ctypes.c_int, [_vp, ctypes.c_char_p])
+_sig("csx_run_sharded_peer", ctypes.c_int, [_vp, _vp, _vp, ctypes.c_int64, _vp])
 _sig("csx_plan_destroy", ctypes.c_int, [_vp])
 _sig("csx_status_string", ctypes.c_char_p, [ctypes.c_int])
 _sig("csx_last_error", ctypes.c_char_p, [])
@@ -84,7 +87,7 @@ _sig("csx_profile_read", ctypes.c_int, [_vp, ctypes.POINTER(ctypes.c_double), _i
 
 _sig("csx_halo_schedule", ctypes.c_int, [_vp, ctypes.c_int, ctypes.c_int, _i64p, ctypes.POINTER(ctypes.c_int)])
 
-EXPORTED = ["csx_auto_fuse_steps", "csx_plan_set_s2r_variant", "csx_halo_schedule", "csx_profile_enable", "csx_profile_read", "csx_plan", "csx_plan_set_engine", "csx_run", "csx_run_host", "csx_comm_create",
+EXPORTED = ["csx_peer_export", "csx_peer_connect", "csx_run_sharded_peer", "csx_auto_fuse_steps", "csx_plan_set_s2r_variant", "csx_halo_schedule", "csx_profile_enable", "csx_profile_read", "csx_plan", "csx_plan_set_engine", "csx_run", "csx_run_host", "csx_comm_create",
             "csx_comm_destroy", "csx_nccl_unique_id", "csx_shard_rows", "csx_run_sharded",
             "csx_plan_destroy", "csx_status_string", "csx_last_error", "csx_plan_info",
             "csx_compose_weights", "csx_weight_matrices", "csx_stencil2row_index",
@@ -273,6 +276,28 @@ def csx_run_sharded(plan, comm, d_in, d_out, timesteps: int, n_local: int, strea
                                 _stream_handle(stream)), "csx_run_sharded")
 
 
+CSX_PEER_DESC_BYTES = 512
+
+
+def csx_peer_export(plan, rank: int, nranks: int) -> bytes:
+    buf = ctypes.create_string_buffer(CSX_PEER_DESC_BYTES)
+    _check(_lib.csx_peer_export(plan, int(rank), int(nranks), buf), "csx_peer_export")
+    return buf.raw
+
+
+def csx_peer_connect(plan, descs):
+    blob = b"".join(descs)
+    if any(len(d) != CSX_PEER_DESC_BYTES for d in descs):
+        raise ValueError("peer descriptors must be CSX_PEER_DESC_BYTES each")
+    _check(_lib.csx_peer_connect(plan, blob), "csx_peer_connect")
+
+
+def csx_run_sharded_peer(plan, d_in, d_out, timesteps: int, n_local: int, stream=None):
+    _check(_lib.csx_run_sharded_peer(plan, _device_ptr(d_in, n_local, "d_in"),
+                                     _device_ptr(d_out, n_local, "d_out"), int(timesteps),
+                                     _stream_handle(stream)), "csx_run_sharded_peer")
+
+
 # ---- owner object ------------------------------------------------------------------------
 class Plan:
     """Owns a csx plan.  ``weights`` is the dense (2r+1)^ndim array (correlation orientation)."""
@@ -323,6 +348,24 @@ class Plan:
 
     def run_sharded(self, comm, d_in, d_out, timesteps: int, n_local: int, stream=None):
         csx_run_sharded(self._h, comm, d_in, d_out, timesteps, n_local, stream)
+
+    def peer_setup(self, rank: int, nranks: int, all_gather=None):
+        """Bootstrap the NVLink peer-memory halo exchange: export this rank's descriptor,
+        all-gather them (default: torch.distributed.all_gather_object on the default group)
+        and connect to the neighbours."""
+        desc = csx_peer_export(self._h, rank, nranks)
+        if nranks == 1:
+            descs = [desc]
+        elif all_gather is not None:
+            descs = all_gather(desc)
+        else:
+            import torch.distributed as dist
+            descs = [None] * nranks
+            dist.all_gather_object(descs, desc)
+        csx_peer_connect(self._h, descs)
+
+    def run_sharded_peer(self, d_in, d_out, timesteps: int, n_local: int, stream=None):
+        csx_run_sharded_peer(self._h, d_in, d_out, timesteps, n_local, stream)
 
     def halo_schedule(self, rank: int, nranks: int):
         return csx_halo_schedule(self._h, rank, nranks)

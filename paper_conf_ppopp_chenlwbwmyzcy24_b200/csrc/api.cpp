@@ -212,6 +212,16 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
         const int64_t need = s2r_explicit_elems(ps.nk, c.E[1], c.E[2]);
         if (need > p->s2r_elems) {
           cudaFree(p->d_s2r);
+    if (p->peer) {
+      csx_peer_s* q = p->peer;
+      for (void* ptr : q->opened) cudaIpcCloseMemHandle(ptr);
+      cudaFree(q->block);
+      if (q->cs) cudaStreamDestroy((cudaStream_t)q->cs);
+      if (q->ev_edge) cudaEventDestroy((cudaEvent_t)q->ev_edge);
+      if (q->ev_x) cudaEventDestroy((cudaEvent_t)q->ev_x);
+      delete q;
+      p->peer = nullptr;
+    }
           p->d_s2r = nullptr;
           p->s2r_elems = 0;
           CSX_CUDA(cudaMalloc(&p->d_s2r, (size_t)need * sizeof(double)), "cudaMalloc(stencil2row)");
@@ -498,8 +508,10 @@ csx_status csx_plan_destroy(csx_plan_t p) {
     cudaFree(p->d_buf[1]);
     cudaFree(p->d_wbase);
     cudaFree(p->d_dense);
-    cudaFree(p->d_sbuf[0]);
-    cudaFree(p->d_sbuf[1]);
+    if (!p->peer) {  // (peer plans keep their slab buffers inside the peer block)
+      cudaFree(p->d_sbuf[0]);
+      cudaFree(p->d_sbuf[1]);
+    }
     cudaFree(p->d_s2r);
 
     cudaSetDevice(cur);

@@ -83,6 +83,26 @@ struct Padded {
 
 }  // namespace csx
 
+// NVLink peer-memory halo exchange state of a sharded plan (comm.cpp, kernels_peer.cu).
+struct csx_peer_s {
+  int rank = 0, nranks = 1, up = -1, down = -1;  // neighbours along the slab axis (-1 none)
+  int64_t El = 0, El_up = 0, El_down = 0;         // slab rows owned by this rank / neighbours
+  double* up_buf[2] = {nullptr, nullptr};         // neighbour slab buffers (allocation bases)
+  double* down_buf[2] = {nullptr, nullptr};
+  // local flag block: [0] READY_TOP (written by up), [1] READY_BOTTOM (by down),
+  // [2] FREED_BY_UP (by up), [3] FREED_BY_DOWN (by down), [4] last-CTA counter
+  unsigned long long* flags = nullptr;
+  void* block = nullptr;                          // one allocation: slab buffers 0, 1 + flags
+  unsigned long long* up_flags = nullptr;         // the neighbours' flag blocks (peer memory)
+  unsigned long long* down_flags = nullptr;
+  std::vector<void*> opened;                      // IPC mappings to close
+  unsigned long long epoch = 0;                   // epoch base of the next run
+  void* cs = nullptr;                             // cudaStream_t: push stream
+  void* ev_edge = nullptr;                        // cudaEvent_t
+  void* ev_x = nullptr;
+  bool connected = false;
+};
+
 struct csx_plan_s {
   int ndim = 0;
   int64_t ext[3] = {1, 1, 1};      // user extents (ext[0] slowest), ndim of them valid
@@ -115,6 +135,7 @@ struct csx_plan_s {
   int64_t s_lo = -1, s_hi = -1;
   int s_rank = -1, s_nranks = 0;
   double* d_dense = nullptr;       // csx_run_host staging grid
+  csx_peer_s* peer = nullptr;      // NVLink peer halo exchange (csx_peer_export / _connect)
   // side stream: the FIXED band fix-up of a TC_TILE 2D pass runs concurrently with the pass
   void* side = nullptr;            // cudaStream_t
   void* ev_fork = nullptr;         // cudaEvent_t

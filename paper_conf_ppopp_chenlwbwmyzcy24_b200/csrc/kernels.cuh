@@ -67,6 +67,28 @@ struct DirectArgs {
   int ndim;
 };
 
+// NVLink peer-memory halo push (kernels_peer.cu)
+struct PeerPushArgs {
+  const double* src_first = nullptr;  // this rank's first h slab rows (full padded rows)
+  const double* src_last = nullptr;   // this rank's last h slab rows
+  double* dst_up = nullptr;           // up neighbour's bottom ghost rows (peer memory) or null
+  double* dst_down = nullptr;         // down neighbour's top ghost rows (peer memory) or null
+  int64_t n = 0;                      // doubles per side
+  int vec2 = 0;                       // all four pointers 16-B aligned
+  const unsigned long long* freed_up = nullptr;    // local: up has finished reading ghosts
+  const unsigned long long* freed_down = nullptr;  // local: down has finished reading ghosts
+  unsigned long long wait_v = 0;
+  unsigned long long* ready_up_remote = nullptr;    // up's READY_BOTTOM
+  unsigned long long* ready_down_remote = nullptr;  // down's READY_TOP
+  unsigned long long* freed_up_remote = nullptr;    // up's FREED_BY_DOWN
+  unsigned long long* freed_down_remote = nullptr;  // down's FREED_BY_UP
+  unsigned long long ready_v = 0, freed_v = 0;      // 0 = do not publish
+  unsigned int* counter = nullptr;                  // local last-CTA counter
+};
+cudaError_t launch_peer_push(const PeerPushArgs& a, cudaStream_t st);
+cudaError_t launch_peer_wait(const unsigned long long* ready_top, const unsigned long long* ready_bottom,
+                             unsigned long long v, cudaStream_t st);
+
 // launchers (return cudaError_t of the launch)
 cudaError_t launch_pack(const double* in, View dst, const int64_t* E, cudaStream_t st);
 cudaError_t launch_ghost_fill(View buf, const int64_t* E, const int* real, const int* fill, int H,
