@@ -46,6 +46,9 @@ CONFIGS = {
     "heat2d_10240": ("heat2d", (10240, 10240), 100, "fixed", 0),
     "star2d9p_10240": ("star2d9p", (10240, 10240), 100, "fixed", 0),     # Table 3 extra shapes
     "box2d25p_10240": ("box2d25p", (10240, 10240), 100, "fixed", 0),
+    # C3 "multi-step fused" as BASELINE.json words it: r = 3, Tf = 2 (nk = 13, reading A4/A7)
+    "star2d13p_10240_tf2": ("star2d13p", (10240, 10240), 100, "fixed", 2),
+    "box2d49p_10240_tf2": ("box2d49p", (10240, 10240), 100, "fixed", 2),
 }
 DEFAULT = "box2d9p_10240"
 METRIC = "FP64 GStencils/s"
@@ -171,9 +174,9 @@ def algorithmic_mma(ndim, nk, engine, points, tc_planes):
         k = nk if ndim == 1 else nk * nk
         return points / (8 * sw) * 2 * math.ceil(k / 4) * nf * tc_planes
     if engine == "tc_tile":
-        a, b = (2, 4) if nk == 5 else (4, 2)
-        kc = 4 * math.ceil((b + nk - 1) / 4)
-        return points / 64 * ((a + nk - 1) * kc // 4) * tc_planes
+        # the block shape of smaller K (planner.cpp): 2x4 for nk = 5, 9, 13; 4x2 otherwise
+        kdim = lambda a, b: (a + nk - 1) * 4 * math.ceil((b + nk - 1) / 4)
+        return points / 64 * (min(kdim(4, 2), kdim(2, 4)) // 4) * tc_planes
     return 0.0
 
 

@@ -70,7 +70,8 @@ typedef struct csx_comm_s* csx_comm_t;
  * buffers (weight fragments, LUT, two padded ping-pong grids) are allocated and uploaded at
  * the first csx_run on the then-current device.
  *   ndim 1..3; extents[ndim] >= 2*r*Tf+1 each; radius 1..3; fuse_steps 0 = automatic
- *   (composed window nk = 2*r*Tf+1: 1D nk <= 31 (TC_S2R: <= 15), 2D nk <= 7, 3D Tf = 1)
+ *   (composed window nk = 2*r*Tf+1: 1D nk <= 31 (TC_S2R: <= 15), 2D nk <= 13 (TC_S2R: <= 7),
+ *   3D Tf = 1)
  *   (DESIGN.md "Fusion depth"), else Tf >= 1.  *out receives the plan (caller frees with
  *   csx_plan_destroy).  Errors: INVALID_ARGUMENT (null pointers, bad ndim/radius/extents,
  *   off-axis star weights, non-finite weights), UNSUPPORTED (a combination no engine covers). */

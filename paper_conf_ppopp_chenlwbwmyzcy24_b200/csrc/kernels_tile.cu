@@ -427,6 +427,12 @@ using Tile7c = TileCfg<7, 4, 2, 8, 4, 6, 2, 3, 2>;
 using Tile7d = TileCfg<7, 4, 2, 8, 8, 2, 3, 3, 1, 2>;  // variant 3: 2 CTAs/SM of 6 DMMA warps (64 x 48)
 using Tile7e = TileCfg<7, 4, 2, 8, 8, 2, 4, 2, 1, 2>;  // variant 4: 2 CTAs/SM of 8 DMMA warps (64 x 64)
 
+// fused windows beyond the paper's one N fragment (reading A7): 8 DMMA warps, CTA 64 x 64,
+// 3-stage ring; the K/4 weight fragments (30 / 42 / 56) stay in registers
+using Tile9 = TileCfg<9, 2, 4, 12, 8, 4, 2, 3>;
+using Tile11 = TileCfg<11, 4, 2, 12, 8, 2, 4, 3>;
+using Tile13 = TileCfg<13, 2, 4, 16, 8, 4, 2, 3>;
+
 static int tile_variant() {
   static int v = -1;
   if (v < 0) {
@@ -871,7 +877,7 @@ static cudaError_t launch_tile1d(int nk, const S2RArgs& a, cudaStream_t st) {
 
 bool tile_kernel_exists(int ndim, int nk) {
   return (ndim == 1 && (nk & 1) && nk >= 3 && nk <= 31) ||
-         (ndim == 2 && (nk == 3 || nk == 5 || nk == 7)) || (ndim == 3 && nk == 3);
+         (ndim == 2 && (nk & 1) && nk >= 3 && nk <= 13) || (ndim == 3 && nk == 3);
 }
 
 template <class C>
@@ -935,6 +941,9 @@ cudaError_t launch_tile(int ndim, int nk, const S2RArgs& a, cudaStream_t st) {
   switch (nk) {
     case 3: return v == 2 ? launch_tile_cfg<Tile3c>(a, st) : v ? launch_tile_cfg<Tile3b>(a, st) : launch_tile_cfg<Tile3>(a, st);
     case 5: return v == 2 ? launch_tile_cfg<Tile5c>(a, st) : v ? launch_tile_cfg<Tile5b>(a, st) : launch_tile_cfg<Tile5>(a, st);
+    case 9: return launch_tile_cfg<Tile9>(a, st);
+    case 11: return launch_tile_cfg<Tile11>(a, st);
+    case 13: return launch_tile_cfg<Tile13>(a, st);
     case 7: return v == 4 ? launch_tile_cfg<Tile7e>(a, st) : v == 3 ? launch_tile_cfg<Tile7d>(a, st) : v == 2 ? launch_tile_cfg<Tile7c>(a, st) : v ? launch_tile_cfg<Tile7b>(a, st) : launch_tile_cfg<Tile7>(a, st);
   }
   return cudaErrorNotSupported;

@@ -256,12 +256,14 @@ csx_status build_pass(const csx_plan_s* p, int tf, Pass* out) {
   const int64_t pts = p->E[0] * p->E[1] * p->E[2];
   const int tcp = ndim == 3 ? P.tc_planes : 1;
   P.mma_per_pass = (int64_t)((double)pts / (8.0 * P.sw) * 2 * P.ks * P.nf * tcp + 0.5);
-  // ---------------- TC_TILE geometry (2D and 3D planes, nk <= 7) ----------------
+  // ---------------- TC_TILE geometry (2D nk <= 13, 3D planes nk <= 7) ----------------
   // The same GEMM with the 8 N columns of a DMMA holding an a x b block of outputs (a*b = 8)
   // instead of 1 x (nk+1): K = the (a+nk-1) x (b+nk-1) input region of the block, each region
   // row padded to kc (a multiple of 4) so that every k-slice is 4 consecutive cells of one
   // input row.  Block shape per nk minimises K: nk=3 -> 4x2 (K=24), nk=5 -> 2x4 (K=48),
-  // nk=7 -> 4x2 (K=80) versus the paper's 2*ceil(nk^2/4)*4 = 24 / 56 / 104.
+  // nk=7 -> 4x2 (K=80) versus the paper's 2*ceil(nk^2/4)*4 = 24 / 56 / 104; fused windows
+  // past one N fragment of the paper's layout (reading A7): nk=9 -> 2x4 (K=120), nk=11 -> 4x2
+  // (K=168), nk=13 -> 2x4 (K=224) versus 2*ceil(nk^2/4)*4*nf = 168 / 248 / 344.
   if (ndim == 1) {
     // 1D TC_TILE: the 8 N columns are 8 consecutive outputs, so the weight operand is the banded
     // Toeplitz matrix W[k][n] = w[k - n] (0 <= k - n < nk), K = nk + 7 rounded up to 4.
@@ -278,9 +280,11 @@ csx_status build_pass(const csx_plan_s* p, int tf, Pass* out) {
       }
     P.tile_mma_per_pass = (int64_t)((double)pts / 64.0 * P.tile_ks + 0.5);
   }
-  if (ndim >= 2 && nk <= 7) {
+  if ((ndim == 2 && nk <= 13) || (ndim == 3 && nk <= 7)) {
+    // block shape: the one of 4x2 / 2x4 with the smaller K = (a+nk-1) * kc
+    auto kdim = [nk](int a_, int b_) { return (a_ + nk - 1) * 4 * ((b_ + nk - 1 + 3) / 4); };
     int a = 4, b = 2;
-    if (nk == 5) { a = 2; b = 4; }
+    if (kdim(2, 4) < kdim(4, 2)) { a = 2; b = 4; }
     const int krows = a + nk - 1;
     const int kc = 4 * ((b + nk - 1 + 3) / 4);
     P.tile_ok = 1;
@@ -330,8 +334,10 @@ csx_status build_plan(csx_plan_s* p) {
   // blocks) nk <= 31 — the FIXED band code's 32-lane cone needs 2 r (Tf-1) <= 31.
   if (p->ndim == 1 && nk > 31)
     return fail(CSX_ERR_UNSUPPORTED, "1D: composed window 2*r*Tf+1 must be <= 31");
-  if (p->ndim == 2 && nk > 7)
-    return fail(CSX_ERR_UNSUPPORTED, "2D: composed window 2*r*Tf+1 must be <= 7 (one N fragment)");
+  // 2D: TC_S2R (the paper's layout, one N fragment) takes nk <= 7; TC_TILE and DIRECT nk <= 13
+  // (C3's "multi-step fused" r = 3, Tf = 2 is nk = 13).
+  if (p->ndim == 2 && nk > 13)
+    return fail(CSX_ERR_UNSUPPORTED, "2D: composed window 2*r*Tf+1 must be <= 13");
   if (p->ndim == 3 && p->tf != 1)
     return fail(CSX_ERR_UNSUPPORTED, "3D: only Tf = 1 (reading A4)");
   for (int a = 0; a < 3; ++a)

@@ -78,6 +78,23 @@ def test_parity_fusion_depths_2d(csx, tf, bc, engine):
         assert rel(got, oracle.run(u0, w, bc, T)) <= TOL, (tf, T)
 
 
+@pytest.mark.parametrize("name,tf", [("box2d9p", 4), ("heat2d", 5), ("box2d9p", 6), ("box2d25p", 2),
+                                     ("box2d25p", 3), ("star2d13p", 2), ("box2d49p", 2)])
+@pytest.mark.parametrize("bc", ["fixed", "periodic"])
+@pytest.mark.parametrize("engine", ["tc_tile", "direct"])
+def test_parity_deep_fusion_2d(csx, name, tf, bc, engine):
+    """2D composed windows past the paper's one N fragment (nk = 9, 11, 13; C3's "multi-step
+    fused" r = 3, Tf = 2): several CTA tiles + ragged tails, T with and without a remainder
+    pass, the FIXED band of depth r*Tf recomputed by k_band."""
+    s = synth.SHAPES[name]
+    u0 = synth.grid((150, 203), seed=9)
+    w = synth.random_weights(name)
+    for T in (tf, 2 * tf + 1, 13):
+        got, info = run_gpu(csx, u0, w, s.kind, bc, T, engine=engine, fuse_steps=tf)
+        assert info["fuse_steps"] == tf and info["engine_name"] == engine
+        assert rel(got, oracle.run(u0, w, bc, T)) <= TOL, (name, tf, T, bc, engine)
+
+
 @pytest.mark.parametrize("tf", [1, 2, 3, 5, 7])
 def test_parity_fusion_depths_1d(csx, tf):
     u0 = synth.grid((3000,), seed=6)

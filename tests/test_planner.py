@@ -235,6 +235,27 @@ def test_1d_fusion_limits():
         csx.Plan((4096,), w, fuse_steps=16)
 
 
+def test_2d_fusion_limits():
+    """2D: TC_TILE runs composed windows up to nk = 13 (C3's "multi-step fused" r = 3, Tf = 2)
+    with the block shape of smaller K: nk = 9 -> 2x4 (K = 120), 11 -> 4x2 (168), 13 -> 2x4
+    (224); the paper's layout (TC_S2R, one N fragment) stops at nk = 7; nk = 15 is refused."""
+    ext = (640, 512)
+    pts = ext[0] * ext[1]
+    for name, tf, nk, ks in (("box2d9p", 4, 9, 30), ("box2d9p", 5, 11, 42),
+                             ("box2d49p", 2, 13, 56), ("star2d13p", 2, 13, 56), ("box2d25p", 3, 13, 56)):
+        s = synth.SHAPES[name]
+        p = csx.Plan(ext, synth.physical_weights(name), shape=s.kind, fuse_steps=tf)
+        info = p.info()
+        assert info["nk"] == nk and info["engine_name"] == "tc_tile", name
+        assert info["mma_per_pass"] == pts // 64 * ks, name
+        with pytest.raises(csx.CsxError):
+            p.set_engine("tc_s2r")
+        p.set_engine("direct")
+        p.close()
+    with pytest.raises(csx.CsxError):
+        csx.Plan(ext, synth.physical_weights("box2d9p"), shape="box", fuse_steps=7)
+
+
 def test_auto_fusion_depths():
     cases = {"heat1d": 11, "1d5p": 5, "heat2d": 3, "box2d9p": 3, "star2d13p": 1, "box2d49p": 1,
              "heat3d": 1, "box3d27p": 1}
