@@ -260,6 +260,10 @@ def main():
                          "no dirty bits, IV padding, V full")
     ap.add_argument("--exchange", default="peer", choices=["peer", "nccl"],
                     help="N > 1 halo exchange: SM peer stores over NVLink (default) or NCCL send/recv")
+    ap.add_argument("--decomp", default="slab", choices=["slab", "pencil"],
+                    help="multi-GPU decomposition: slabs along the slowest axis (default) or a "
+                         "p0 x p1 pencil / block grid over the two slowest axes (NCCL exchange; "
+                         "--gpus 1 runs the 1 x 1 pencil path)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-comparator", action="store_true")
@@ -306,7 +310,15 @@ def main():
     shape, ext, T, bc, tf = CONFIGS[args.config]
     s = synth.SHAPES[shape]
     w = synth.physical_weights(shape)
-    gext = (ext[0] * world,) + tuple(ext[1:])  # weak scaling: ext per GPU
+    pencil = args.decomp == "pencil"
+    if pencil:
+        if s.ndim < 2:
+            raise SystemExit("--decomp pencil needs a 2D or 3D shape")
+        p1 = max(d for d in range(1, int(math.isqrt(world)) + 1) if world % d == 0)
+        p0 = world // p1
+        gext = (ext[0] * p0, ext[1] * p1) + tuple(ext[2:])  # weak scaling: ext per GPU
+    else:
+        gext = (ext[0] * world,) + tuple(ext[1:])  # weak scaling: ext per GPU
     plan = csx.Plan(gext, w, shape=s.kind, bc=bc, fuse_steps=tf, engine=args.engine)
     if args.s2r_variant == "I":
         plan.set_s2r_variant(padding=3, dirty_bits=True)
@@ -319,7 +331,15 @@ def main():
     stream = torch.cuda.current_stream()
     comm = None
     exchange = None
-    if world > 1:
+    if pencil:
+        exchange = f"nccl pencil {p0}x{p1}"
+        uid = [csx.csx_nccl_unique_id() if rank == 0 else None]
+        if world > 1:
+            dist.broadcast_object_list(uid, src=0)
+        comm = csx.csx_comm_create(uid[0], rank, world)
+        lo, hi = plan.shard_box(rank, p0, p1)
+        u0 = np.ascontiguousarray(synth.grid(gext, rows=(lo[0], hi[0]))[:, lo[1]:hi[1]])
+    elif world > 1:
         exchange = args.exchange
         if exchange == "peer":
             # halo exchange by SM peer stores over NVLink (CUDA IPC), epoch flags in peer memory;
@@ -345,14 +365,16 @@ def main():
             comm = csx.csx_comm_create(uid[0], rank, world)
         lo, hi = plan.shard_rows(rank, world)
         u0 = synth.grid(gext, rows=(lo, hi))
-    else:
+    if not pencil and world == 1:
         u0 = synth.grid(gext)
     d_in = torch.from_numpy(u0).cuda()
     d_out = torch.empty_like(d_in)
     n_local = u0.size
 
     def step():
-        if world == 1:
+        if pencil:
+            plan.run_sharded_pencil(comm, p0, p1, d_in, d_out, T, n_local, stream)
+        elif world == 1:
             plan.run(d_in, d_out, T, stream)
         elif comm is None:
             plan.run_sharded_peer(d_in, d_out, T, n_local, stream)
@@ -444,7 +466,7 @@ def main():
             "config": {"workload": args.config, "shape": shape, "grid": list(gext), "T": T, "bc": bc,
                        "fuse_steps": tfm, "nk": nk, "engine": engine,
                        "s2r_variant": args.s2r_variant if engine == "tc_s2r" else None,
-                       "parallelism": f"slab{world}" if world > 1 else "single",
+                       "parallelism": (f"pencil{p0}x{p1}" if pencil else f"slab{world}" if world > 1 else "single"),
                        "exchange": exchange,
                        "l2": ("L2 flushed (256 MB write) between timed steps" if flush is not None
                               else f"inputs larger than L2 ({u0.nbytes >> 20} MB per grid vs 126 MB); no flush")},

@@ -137,6 +137,28 @@ csx_status csx_halo_schedule(const csx_plan_t plan, int rank, int nranks, int64_
 csx_status csx_run_sharded(csx_plan_t plan, csx_comm_t comm, const double* d_in_local,
                            double* d_out_local, int64_t timesteps, void* stream);
 
+/* ----- Pencil (block) decomposition (not in the paper) -------------
+ * The two slowest stencil axes are split over a p0 x p1 process grid (p0 * p1 = nranks):
+ * 3D (z, y) — every rank owns a pencil running the full x extent; 2D (rows, cols) — blocks.
+ * rank = i0 * p1 + i1 owns [floor(i0 N_a / p0), floor((i0+1) N_a / p0)) along the first split
+ * axis and the same with (i1, p1, N_b) along the second.  Halos of depth r*Tf are exchanged in
+ * two phases per pass (second split axis first, packed strided faces; then the first split axis
+ * with full padded rows, which carry the corners / edges).  Not overlapped with compute.
+ *
+ * csx_shard_box: lo[ndim], hi[ndim] of rank's block in the user's axis order.
+ * csx_pencil_schedule: up to 8 ops of 5 int64 {phase (0 second split axis, 1 first), kind
+ *   (0 send, 1 recv), peer rank, first row along the phase's axis (local index; negative = low
+ *   ghosts, >= local extent = high ghosts), rows (= r*Tf)} in posting order; *nops = count.
+ * csx_run_sharded_pencil: d_in_local / d_out_local hold rank's block (dense, C order); every
+ *   rank calls with equal plan parameters, p0, p1 and T.  INVALID_ARGUMENT if p0*p1 differs
+ *   from the communicator size; UNSUPPORTED for ndim = 1 or a block thinner than r*Tf. */
+csx_status csx_shard_box(const csx_plan_t plan, int rank, int p0, int p1, int64_t* lo, int64_t* hi);
+csx_status csx_pencil_schedule(const csx_plan_t plan, int rank, int p0, int p1, int64_t* ops,
+                               int* nops);
+csx_status csx_run_sharded_pencil(csx_plan_t plan, csx_comm_t comm, int p0, int p1,
+                                  const double* d_in_local, double* d_out_local, int64_t timesteps,
+                                  void* stream);
+
 /* ----- Slab halo exchange over NVLink peer memory (no NCCL on the data path) -----------
  * The same slab decomposition and results as csx_run_sharded, but after every pass the
  * boundary slab rows are copied by SM peer stores straight into the neighbours' ghost rows

@@ -86,8 +86,13 @@ _sig("csx_profile_enable", ctypes.c_int, [_vp, ctypes.c_int])
 _sig("csx_profile_read", ctypes.c_int, [_vp, ctypes.POINTER(ctypes.c_double), _i64p, _i64p, ctypes.c_int])
 
 _sig("csx_halo_schedule", ctypes.c_int, [_vp, ctypes.c_int, ctypes.c_int, _i64p, ctypes.POINTER(ctypes.c_int)])
+_sig("csx_shard_box", ctypes.c_int, [_vp, ctypes.c_int, ctypes.c_int, ctypes.c_int, _i64p, _i64p])
+_sig("csx_pencil_schedule", ctypes.c_int, [_vp, ctypes.c_int, ctypes.c_int, ctypes.c_int, _i64p,
+                                           ctypes.POINTER(ctypes.c_int)])
+_sig("csx_run_sharded_pencil", ctypes.c_int, [_vp, _vp, ctypes.c_int, ctypes.c_int, _vp, _vp,
+                                              ctypes.c_int64, _vp])
 
-EXPORTED = ["csx_peer_export", "csx_peer_connect", "csx_run_sharded_peer", "csx_auto_fuse_steps", "csx_plan_set_s2r_variant", "csx_halo_schedule", "csx_profile_enable", "csx_profile_read", "csx_plan", "csx_plan_set_engine", "csx_run", "csx_run_host", "csx_comm_create",
+EXPORTED = ["csx_shard_box", "csx_pencil_schedule", "csx_run_sharded_pencil", "csx_peer_export", "csx_peer_connect", "csx_run_sharded_peer", "csx_auto_fuse_steps", "csx_plan_set_s2r_variant", "csx_halo_schedule", "csx_profile_enable", "csx_profile_read", "csx_plan", "csx_plan_set_engine", "csx_run", "csx_run_host", "csx_comm_create",
             "csx_comm_destroy", "csx_nccl_unique_id", "csx_shard_rows", "csx_run_sharded",
             "csx_plan_destroy", "csx_status_string", "csx_last_error", "csx_plan_info",
             "csx_compose_weights", "csx_weight_matrices", "csx_stencil2row_index",
@@ -276,6 +281,34 @@ def csx_run_sharded(plan, comm, d_in, d_out, timesteps: int, n_local: int, strea
                                 _stream_handle(stream)), "csx_run_sharded")
 
 
+def csx_shard_box(plan, rank: int, p0: int, p1: int):
+    """([lo per axis], [hi per axis]) of rank's block on the p0 x p1 process grid."""
+    lo = np.zeros(3, dtype=np.int64)
+    hi = np.zeros(3, dtype=np.int64)
+    _check(_lib.csx_shard_box(plan, rank, p0, p1, lo.ctypes.data_as(_i64p), hi.ctypes.data_as(_i64p)),
+           "csx_shard_box")
+    nd = int(csx_plan_info(plan)["ndim"])
+    return [int(v) for v in lo[:nd]], [int(v) for v in hi[:nd]]
+
+
+def csx_pencil_schedule(plan, rank: int, p0: int, p1: int):
+    """[(phase 0 (second split axis) | 1 (first split axis), 'send'|'recv', peer, first_row,
+    nrows), ...] in posting order."""
+    ops = np.zeros(40, dtype=np.int64)
+    n = ctypes.c_int()
+    _check(_lib.csx_pencil_schedule(plan, rank, p0, p1, ops.ctypes.data_as(_i64p), ctypes.byref(n)),
+           "csx_pencil_schedule")
+    return [(int(ops[5 * k]), "send" if ops[5 * k + 1] == 0 else "recv", int(ops[5 * k + 2]),
+             int(ops[5 * k + 3]), int(ops[5 * k + 4])) for k in range(n.value)]
+
+
+def csx_run_sharded_pencil(plan, comm, p0: int, p1: int, d_in, d_out, timesteps: int, n_local: int,
+                           stream=None):
+    _check(_lib.csx_run_sharded_pencil(plan, comm, int(p0), int(p1), _device_ptr(d_in, n_local, "d_in"),
+                                       _device_ptr(d_out, n_local, "d_out"), int(timesteps),
+                                       _stream_handle(stream)), "csx_run_sharded_pencil")
+
+
 CSX_PEER_DESC_BYTES = 512
 
 
@@ -369,6 +402,16 @@ class Plan:
 
     def halo_schedule(self, rank: int, nranks: int):
         return csx_halo_schedule(self._h, rank, nranks)
+
+    def shard_box(self, rank: int, p0: int, p1: int):
+        return csx_shard_box(self._h, rank, p0, p1)
+
+    def pencil_schedule(self, rank: int, p0: int, p1: int):
+        return csx_pencil_schedule(self._h, rank, p0, p1)
+
+    def run_sharded_pencil(self, comm, p0: int, p1: int, d_in, d_out, timesteps: int, n_local: int,
+                           stream=None):
+        csx_run_sharded_pencil(self._h, comm, p0, p1, d_in, d_out, timesteps, n_local, stream)
 
     def lut(self):
         return csx_plan_lut(self._h)

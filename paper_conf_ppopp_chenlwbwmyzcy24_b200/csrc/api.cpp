@@ -212,6 +212,7 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
         const int64_t need = s2r_explicit_elems(ps.nk, c.E[1], c.E[2]);
         if (need > p->s2r_elems) {
           cudaFree(p->d_s2r);
+    cudaFree(p->d_pstage);
     if (p->peer) {
       csx_peer_s* q = p->peer;
       for (void* ptr : q->opened) cudaIpcCloseMemHandle(ptr);
@@ -513,6 +514,7 @@ csx_status csx_plan_destroy(csx_plan_t p) {
       cudaFree(p->d_sbuf[1]);
     }
     cudaFree(p->d_s2r);
+    cudaFree(p->d_pstage);
 
     cudaSetDevice(cur);
   }

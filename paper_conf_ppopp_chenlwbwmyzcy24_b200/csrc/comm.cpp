@@ -191,7 +191,7 @@ static csx_status run_sharded_impl(csx_plan_s* p, csx_comm_s* c, csx_peer_s* q, 
   if (q) {
     if (p->s_rank != rank || p->s_nranks != nranks || !p->d_sbuf[0])
       return fail(CSX_ERR_INTERNAL, "peer slab buffers changed after export");
-  } else if (p->s_rank != rank || p->s_nranks != nranks) {
+  } else if (p->s_rank != rank || p->s_nranks != nranks || p->s_p1 != 0) {
     cudaFree(p->d_sbuf[0]);
     cudaFree(p->d_sbuf[1]);
     p->d_sbuf[0] = p->d_sbuf[1] = nullptr;
@@ -199,6 +199,7 @@ static csx_status run_sharded_impl(csx_plan_s* p, csx_comm_s* c, csx_peer_s* q, 
     if (s != CSX_OK) return s;
     p->s_rank = rank;
     p->s_nranks = nranks;
+    p->s_p0 = p->s_p1 = 0;
     p->s_lo = lo;
     p->s_hi = hi;
   }
@@ -307,6 +308,250 @@ static csx_status run_sharded_impl(csx_plan_s* p, csx_comm_s* c, csx_peer_s* q, 
   return CSX_OK;
 }
 
+
+// ---- Pencil (block) decomposition over a p0 x p1 process grid ----------
+//
+// The two slowest stencil axes are split: 3D (z, y) — every rank owns a pencil running the full
+// x extent; 2D (rows, cols) — blocks.  Rank = i0 * p1 + i1 owns [lo, hi) along axis a (index
+// i0 of p0) and axis b (i1 of p1), floor partitions as for slabs.  Ghosts (depth r*Tf) are
+// exchanged in two phases per pass, so that corners (edges in 3D) travel through the face
+// neighbours: phase 0 along axis b for the owned range of axis a (strided faces, packed into a
+// contiguous staging buffer by cudaMemcpy2DAsync around the NCCL group); phase 1 along axis a
+// with full padded rows of axis b — which now include the axis-b ghosts just received.
+
+#define COMM_CUDA(call, where)                  \
+  do {                                          \
+    cudaError_t e_ = (call);                    \
+    if (e_ != cudaSuccess) return cuda_fail(e_, where); \
+  } while (0)
+
+static void pencil_axes(const csx_plan_s* p, int* aa, int* ab) {
+  *aa = p->ndim == 3 ? 0 : 1;
+  *ab = *aa + 1;
+}
+
+static void pencil_box(const csx_plan_s* p, int rank, int p0, int p1, int64_t* lo, int64_t* hi) {
+  int aa, ab;
+  pencil_axes(p, &aa, &ab);
+  for (int a = 0; a < 3; ++a) { lo[a] = 0; hi[a] = p->E[a]; }
+  const int i0 = rank / p1, i1 = rank - (rank / p1) * p1;
+  lo[aa] = (int64_t)i0 * p->E[aa] / p0;
+  hi[aa] = (int64_t)(i0 + 1) * p->E[aa] / p0;
+  lo[ab] = (int64_t)i1 * p->E[ab] / p1;
+  hi[ab] = (int64_t)(i1 + 1) * p->E[ab] / p1;
+}
+
+// ops of 5 int64: {phase (0 axis b, 1 axis a), kind (0 send, 1 recv), peer, first row along the
+// phase's axis (local interior index; negative = low ghosts, >= local extent = high ghosts), rows}.
+// Per phase the slab order: send high rows to the high neighbour, recv low ghosts from the low
+// one, send low rows to the low neighbour, recv high ghosts from the high one.
+static int pencil_schedule(const csx_plan_s* p, int rank, int p0, int p1, const int64_t* El, int64_t* ops) {
+  int aa, ab;
+  pencil_axes(p, &aa, &ab);
+  const int h = p->halo;
+  const bool periodic = p->bc == CSX_BC_PERIODIC;
+  const int i0 = rank / p1, i1 = rank - (rank / p1) * p1;
+  int n = 0;
+  for (int phase = 0; phase < 2; ++phase) {
+    const int np = phase == 0 ? p1 : p0, me = phase == 0 ? i1 : i0;
+    const int64_t Ex = El[phase == 0 ? ab : aa];
+    auto peer_of = [&](int idx) { return phase == 0 ? i0 * p1 + idx : idx * p1 + i1; };
+    int lo_n = me - 1, hi_n = me + 1;
+    if (periodic) {
+      lo_n = (lo_n + np) % np;
+      hi_n = hi_n % np;
+    } else {
+      if (lo_n < 0) lo_n = -1;
+      if (hi_n >= np) hi_n = -1;
+    }
+    auto op = [&](int kind, int peer, int64_t row) {
+      int64_t* o = ops + 5 * n++;
+      o[0] = phase; o[1] = kind; o[2] = peer; o[3] = row; o[4] = h;
+    };
+    if (hi_n >= 0) op(0, peer_of(hi_n), Ex - h);
+    if (lo_n >= 0) { op(1, peer_of(lo_n), -h); op(0, peer_of(lo_n), 0); }
+    if (hi_n >= 0) op(1, peer_of(hi_n), Ex);
+  }
+  return n;
+}
+
+// A face of h rows along axis b (phase 0) as a 2D copy: `height` runs of `width` contiguous
+// doubles, `pitch` apart.  3D (b = y): one run per z plane of the owned range, h padded rows
+// each; 2D (b = cols): one run per owned row, h cells each.
+static void face_b(const csx_plan_s* p, const Padded& pd, double* base, int64_t row, int h,
+                   const int64_t* El, double** ptr, size_t* width, size_t* height, size_t* pitch) {
+  if (p->ndim == 3) {
+    *ptr = base + pd.O[0] * pd.s0 + (pd.O[1] + row) * pd.s1;
+    *width = (size_t)h * pd.s1;
+    *height = (size_t)El[0];
+    *pitch = (size_t)pd.s0;
+  } else {
+    *ptr = base + pd.O[1] * pd.s1 + pd.O[2] + row;
+    *width = (size_t)h;
+    *height = (size_t)El[1];
+    *pitch = (size_t)pd.s1;
+  }
+}
+
+static csx_status exchange_pencil(csx_plan_s* p, csx_comm_s* c, double* base, int p0, int p1,
+                                  const int64_t* El, cudaStream_t st) {
+  int64_t ops[40];
+  const int nops = pencil_schedule(p, c->rank, p0, p1, El, ops);
+  int aa, ab;
+  pencil_axes(p, &aa, &ab);
+  const Padded& pd = p->spad;
+  for (int phase = 0; phase < 2; ++phase) {
+    size_t stage_off = 0;
+    // phase 0: pack the strided send faces
+    if (phase == 0)
+      for (int k = 0; k < nops; ++k) {
+        const int64_t* o = ops + 5 * k;
+        if (o[0] != 0) continue;
+        double* ptr;
+        size_t w, hgt, pitch;
+        face_b(p, pd, base, o[3], (int)o[4], El, &ptr, &w, &hgt, &pitch);
+        if (o[1] == 0)
+          COMM_CUDA(cudaMemcpy2DAsync(p->d_pstage + stage_off, w * 8, ptr, pitch * 8, w * 8, hgt,
+                                     cudaMemcpyDeviceToDevice, st), "pack face");
+        stage_off += w * hgt;
+      }
+    ncclResult_t r = ncclGroupStart();
+    if (r != ncclSuccess) return nccl_fail(r, "ncclGroupStart");
+    stage_off = 0;
+    for (int k = 0; k < nops; ++k) {
+      const int64_t* o = ops + 5 * k;
+      if (o[0] != phase) continue;
+      double* ptr;
+      size_t n;
+      if (phase == 0) {
+        size_t w, hgt, pitch;
+        face_b(p, pd, base, o[3], (int)o[4], El, &ptr, &w, &hgt, &pitch);
+        ptr = p->d_pstage + stage_off;
+        n = w * hgt;
+        stage_off += n;
+      } else {
+        slab_rows(pd, base, aa, o[3], (int)o[4], &ptr, &n);
+      }
+      if (o[1] == 0) r = ncclSend(ptr, n, ncclDouble, (int)o[2], c->comm, st);
+      else r = ncclRecv(ptr, n, ncclDouble, (int)o[2], c->comm, st);
+      if (r != ncclSuccess) return nccl_fail(r, o[1] == 0 ? "ncclSend" : "ncclRecv");
+    }
+    r = ncclGroupEnd();
+    if (r != ncclSuccess) return nccl_fail(r, "ncclGroupEnd");
+    // phase 0: unpack the received faces into the axis-b ghosts
+    if (phase == 0) {
+      stage_off = 0;
+      for (int k = 0; k < nops; ++k) {
+        const int64_t* o = ops + 5 * k;
+        if (o[0] != 0) continue;
+        double* ptr;
+        size_t w, hgt, pitch;
+        face_b(p, pd, base, o[3], (int)o[4], El, &ptr, &w, &hgt, &pitch);
+        if (o[1] == 1)
+          COMM_CUDA(cudaMemcpy2DAsync(ptr, pitch * 8, p->d_pstage + stage_off, w * 8, w * 8, hgt,
+                                     cudaMemcpyDeviceToDevice, st), "unpack face");
+        stage_off += w * hgt;
+      }
+    }
+  }
+  return CSX_OK;
+}
+
+static csx_status run_sharded_pencil_impl(csx_plan_s* p, csx_comm_s* c, int p0, int p1,
+                                          const double* d_in, double* d_out, int64_t T,
+                                          cudaStream_t st) {
+  if (T < 0) return fail(CSX_ERR_INVALID_ARGUMENT, "timesteps < 0");
+  if (p->ndim < 2) return fail(CSX_ERR_UNSUPPORTED, "pencil decomposition needs ndim >= 2");
+  if (p0 < 1 || p1 < 1 || p0 * p1 != c->nranks)
+    return fail(CSX_ERR_INVALID_ARGUMENT, "process grid p0 x p1 must equal the communicator size");
+  const int rank = c->rank, nranks = c->nranks;
+  int aa, ab;
+  pencil_axes(p, &aa, &ab);
+  int64_t lo[3], hi[3], El[3];
+  pencil_box(p, rank, p0, p1, lo, hi);
+  for (int a = 0; a < 3; ++a) El[a] = hi[a] - lo[a];
+  if (El[aa] < p->halo || El[ab] < p->halo || El[aa] < 1 || El[ab] < 1)
+    return fail(CSX_ERR_UNSUPPORTED, "a rank owns fewer rows than the halo depth r*Tf along a split axis");
+  const int64_t n = El[0] * El[1] * El[2];
+  csx_status s = ensure_device(p);
+  if (s != CSX_OK) return s;
+  if (T == 0) {
+    if (d_in != d_out) {
+      cudaError_t e = cudaMemcpyAsync(d_out, d_in, n * sizeof(double), cudaMemcpyDeviceToDevice, st);
+      if (e != cudaSuccess) return cuda_fail(e, "copy");
+    }
+    return CSX_OK;
+  }
+  if (p->peer) return fail(CSX_ERR_INVALID_ARGUMENT, "plan is bound to a peer slab exchange");
+  if (p->s_rank != rank || p->s_nranks != nranks || p->s_p0 != p0 || p->s_p1 != p1) {
+    cudaFree(p->d_sbuf[0]);
+    cudaFree(p->d_sbuf[1]);
+    p->d_sbuf[0] = p->d_sbuf[1] = nullptr;
+    s = ensure_grid(p, &p->spad, p->d_sbuf, El);
+    if (s != CSX_OK) return s;
+    p->s_rank = rank;
+    p->s_nranks = nranks;
+    p->s_p0 = p0;
+    p->s_p1 = p1;
+    p->s_lo = lo[aa];
+    p->s_hi = hi[aa];
+  }
+  const Padded& pd = p->spad;
+  // staging: the 4 phase-0 faces (2 send, 2 recv) of h rows each
+  {
+    double* ptr;
+    size_t w, hgt, pitch;
+    face_b(p, pd, p->d_sbuf[0], 0, p->halo, El, &ptr, &w, &hgt, &pitch);
+    const size_t need = 4 * w * hgt;
+    if (need > p->pstage_elems) {
+      cudaFree(p->d_pstage);
+      p->d_pstage = nullptr;
+      p->pstage_elems = 0;
+      COMM_CUDA(cudaMalloc(&p->d_pstage, need * sizeof(double)), "cudaMalloc(pencil staging)");
+      p->pstage_elems = need;
+    }
+  }
+  const int real[3] = {p->ndim == 3, p->ndim >= 2, 1};
+  int fill[3] = {real[0], real[1], real[2]};
+  fill[aa] = fill[ab] = 0;  // the split axes are filled by the exchange
+  View b[2];
+  for (int i = 0; i < 2; ++i) b[i] = View{p->d_sbuf[i] + pd.origin(), pd.s0, pd.s1};
+  cudaError_t e = launch_pack(d_in, b[0], El, st);
+  if (e != cudaSuccess) return cuda_fail(e, "pack");
+  p->n_launches += 1;
+  auto ghosts = [&](int i) -> csx_status {
+    if (p->bc == CSX_BC_PERIODIC && (fill[0] || fill[1] || fill[2])) {
+      cudaError_t e2 = launch_ghost_fill(b[i], El, real, fill, p->halo, st);
+      if (e2 != cudaSuccess) return cuda_fail(e2, "ghost fill");
+      p->n_launches += fill[0] + fill[1] + fill[2];
+    }
+    return exchange_pencil(p, c, p->d_sbuf[i], p0, p1, El, st);
+  };
+  const int64_t nmain = T / p->tf;
+  const int rem = (int)(T % p->tf);
+  const int64_t npass = nmain + (rem ? 1 : 0);
+  s = ghosts(0);
+  if (s != CSX_OK) return s;
+  const View out{d_out, El[1] * El[2], El[2]};
+  int cur = 0;
+  for (int64_t i = 0; i < npass; ++i) {
+    const int tfp = i < nmain ? p->tf : rem;
+    const bool last = i == npass - 1;
+    PassCtx pc;
+    pc.src = CView{b[cur].p, b[cur].s0, b[cur].s1, pd.O[0], pd.O[1], pd.O[2], pd.A[0]};
+    pc.dst = last ? out : b[cur ^ 1];
+    for (int a = 0; a < 3; ++a) { pc.E[a] = El[a]; pc.gorg[a] = lo[a]; }
+    s = run_pass(p, p->passes[tfp - 1], pc, st);
+    if (s != CSX_OK) return s;
+    if (!last) {
+      s = ghosts(cur ^ 1);
+      if (s != CSX_OK) return s;
+    }
+    cur ^= 1;
+  }
+  return CSX_OK;
+}
+
 }  // namespace csx
 
 using namespace csx;
@@ -381,6 +626,36 @@ csx_status csx_run_sharded(csx_plan_t p, csx_comm_t c, const double* d_in, doubl
                            int64_t T, void* stream) {
   if (!p || !c || !d_in || !d_out) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL argument");
   return run_sharded_impl(p, c, nullptr, d_in, d_out, T, reinterpret_cast<cudaStream_t>(stream));
+}
+
+csx_status csx_shard_box(const csx_plan_t p, int rank, int p0, int p1, int64_t* lo, int64_t* hi) {
+  if (!p || !lo || !hi || p0 < 1 || p1 < 1 || rank < 0 || rank >= p0 * p1)
+    return fail(CSX_ERR_INVALID_ARGUMENT, "bad shard arguments");
+  if (p->ndim < 2) return fail(CSX_ERR_UNSUPPORTED, "pencil decomposition needs ndim >= 2");
+  int64_t l3[3], h3[3];
+  pencil_box(p, rank, p0, p1, l3, h3);
+  for (int a = 0; a < p->ndim; ++a) {  // user axis order: axis a of ndim = normalised 3 - ndim + a
+    lo[a] = l3[3 - p->ndim + a];
+    hi[a] = h3[3 - p->ndim + a];
+  }
+  return CSX_OK;
+}
+
+csx_status csx_pencil_schedule(const csx_plan_t p, int rank, int p0, int p1, int64_t* ops, int* nops) {
+  if (!p || !ops || !nops || p0 < 1 || p1 < 1 || rank < 0 || rank >= p0 * p1)
+    return fail(CSX_ERR_INVALID_ARGUMENT, "bad arguments");
+  if (p->ndim < 2) return fail(CSX_ERR_UNSUPPORTED, "pencil decomposition needs ndim >= 2");
+  int64_t lo[3], hi[3], El[3];
+  pencil_box(p, rank, p0, p1, lo, hi);
+  for (int a = 0; a < 3; ++a) El[a] = hi[a] - lo[a];
+  *nops = pencil_schedule(p, rank, p0, p1, El, ops);
+  return CSX_OK;
+}
+
+csx_status csx_run_sharded_pencil(csx_plan_t p, csx_comm_t c, int p0, int p1, const double* d_in,
+                                  double* d_out, int64_t T, void* stream) {
+  if (!p || !c || !d_in || !d_out) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL argument");
+  return run_sharded_pencil_impl(p, c, p0, p1, d_in, d_out, T, reinterpret_cast<cudaStream_t>(stream));
 }
 
 csx_status csx_run_sharded_peer(csx_plan_t p, const double* d_in, double* d_out, int64_t T,

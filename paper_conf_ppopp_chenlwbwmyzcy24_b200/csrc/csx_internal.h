@@ -134,6 +134,9 @@ struct csx_plan_s {
   double* d_halo = nullptr;        // 4 halo staging slabs (send lo/hi, recv lo/hi)
   int64_t s_lo = -1, s_hi = -1;
   int s_rank = -1, s_nranks = 0;
+  int s_p0 = 0, s_p1 = 0;          // pencil process grid of the sharded buffers (0: slabs)
+  double* d_pstage = nullptr;      // pencil halo staging (4 strided faces packed contiguously)
+  size_t pstage_elems = 0;
   double* d_dense = nullptr;       // csx_run_host staging grid
   csx_peer_s* peer = nullptr;      // NVLink peer halo exchange (csx_peer_export / _connect)
   // side stream: the FIXED band fix-up of a TC_TILE 2D pass runs concurrently with the pass

@@ -21,4 +21,6 @@ cap box3d27p_tc_tile k_tile3d 3 --config box3d27p_512
 cap heat3d_tc_tile k_tile3d 3 --config heat3d_512
 cap heat1d_tc_tile k_tile1d 5 --config heat1d_10240000
 cap box2d49p_tc_tile k_tile2d 3 --config box2d49p_10240
+cap box2d49p_tf2_tc_tile k_tile2d 3 --config box2d49p_10240_tf2
+cap 1d5p_tc_tile k_tile1d 5 --config 1d5p_10240000
 ls -la gpurun_out/$TAG

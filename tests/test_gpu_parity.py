@@ -284,3 +284,32 @@ def test_sharded_overlap_schedule(csx, monkeypatch, name, ext, T, bc):
     csx.csx_comm_destroy(comm)
     p.close()
     assert rel(d_out.cpu().numpy(), oracle.run(u0, w, bc, T)) <= TOL, (name, bc)
+
+
+@pytest.mark.parametrize("name,ext,T", [("box2d9p", (200, 150), 7), ("heat3d", (40, 33, 50), 3),
+                                        ("box3d27p", (21, 40, 35), 2), ("box2d49p", (90, 70), 3)])
+@pytest.mark.parametrize("bc", ["fixed", "periodic"])
+def test_sharded_pencil_single_rank(csx, name, ext, T, bc):
+    """csx_run_sharded_pencil on a 1 x 1 process grid: the two-phase face exchange runs through
+    NCCL (PERIODIC: self send/recv of packed strided faces + full padded rows), then the same pass
+    kernels; equal to the oracle."""
+    s = synth.SHAPES[name]
+    w = synth.random_weights(name)
+    u0 = synth.grid(ext, seed=15)
+    p = csx.Plan(u0.shape, w, shape=s.kind, bc=bc)
+    comm = csx.csx_comm_create(csx.csx_nccl_unique_id(), 0, 1)
+    d_in = torch.from_numpy(u0).cuda()
+    d_out = torch.empty_like(d_in)
+    with pytest.raises(csx.CsxError):
+        p.run_sharded_pencil(comm, 2, 1, d_in, d_out, T, u0.size)  # grid != communicator size
+    p.run_sharded_pencil(comm, 1, 1, d_in, d_out, T, u0.size)
+    torch.cuda.synchronize()
+    got = d_out.cpu().numpy()
+    p.run_sharded(comm, d_in, d_out, T, u0.size)  # back to slabs on the same plan
+    torch.cuda.synchronize()
+    got_slab = d_out.cpu().numpy()
+    csx.csx_comm_destroy(comm)
+    p.close()
+    ref = oracle.run(u0, w, bc, T)
+    assert rel(got, ref) <= TOL, (name, bc)
+    assert rel(got_slab, ref) <= TOL, (name, bc)
