@@ -266,6 +266,10 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
     d.ntiles = (int64_t)d.tiles[0] * d.tiles[1] * d.tiles[2];
     if (p->ndim == 2 && direct2d_exists(p->radius, ps.tf))
       e = launch_direct2d(d, p->w.data(), st);
+    else if (p->ndim == 1 && direct1d_exists(p->radius, ps.tf) && !getenv("CSX_DIRECT_GENERIC"))
+      e = launch_direct1d(d, p->w.data(), st);
+    else if (p->ndim == 3 && direct3d_exists(p->radius, ps.tf) && !getenv("CSX_DIRECT_GENERIC"))
+      e = launch_direct3d(d, p->w.data(), st);
     else
       e = launch_direct(d, st);
     if (e != cudaSuccess) return cuda_fail(e, "direct launch");

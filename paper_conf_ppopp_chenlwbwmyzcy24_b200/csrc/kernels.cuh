@@ -99,6 +99,11 @@ cudaError_t launch_direct(const DirectArgs& a, cudaStream_t st);
 // 2D comparator kernel (kernels_direct2d.cu): compile-time (r, Tf), weights by value.
 bool direct2d_exists(int r, int tf);
 cudaError_t launch_direct2d(const DirectArgs& a, const double* w_host, cudaStream_t st);
+// 1D / 3D comparator kernels (kernels_direct13.cu): compile-time r, weights by value.
+bool direct1d_exists(int r, int tf);
+cudaError_t launch_direct1d(const DirectArgs& a, const double* w_host, cudaStream_t st);
+bool direct3d_exists(int r, int tf);
+cudaError_t launch_direct3d(const DirectArgs& a, const double* w_host, cudaStream_t st);
 // FIXED band fix-up after a fused pass of Tf > 1 steps (kernels_band.cu), 1D and 2D.
 cudaError_t launch_band(int ndim, int r, int tf, CView src, View dst, const int64_t* E,
                         const int64_t* gorg, const int64_t* GE, const double* w_host,

@@ -245,6 +245,30 @@ def test_direct_comparator_2d_all_radii(csx):
             assert rel(got, oracle.run(u0, w, bc, 9)) <= TOL, (r, tf, bc)
 
 
+@pytest.mark.parametrize("generic", [False, True])
+def test_direct_comparator_1d_3d(csx, monkeypatch, generic):
+    """The 1D (register window + shuffles, Tf fused) and 3D (z-march, cp.async plane ring)
+    comparator kernels, and the generic smem kernel they replace (CSX_DIRECT_GENERIC=1), for
+    r = 1..3, several fusion depths, ragged extents, both boundaries, signed weights."""
+    if generic:
+        monkeypatch.setenv("CSX_DIRECT_GENERIC", "1")
+    cases = [(1, 1, 1, (9001,), 13), (1, 1, 11, (20000,), 25), (1, 2, 5, (7777,), 12),
+             (1, 3, 5, (4099,), 11), (1, 1, 15, (3000,), 33),
+             (3, 1, 1, (37, 45, 70), 3), (3, 2, 1, (19, 33, 130), 2), (3, 3, 1, (16, 40, 66), 2)]
+    for ndim, r, tf, ext, T in cases:
+        w = synth.random_signed_weights(ndim, r, seed=60 + r)
+        u0 = synth.grid(ext, seed=61)
+        for bc in ("fixed", "periodic"):
+            got, info = run_gpu(csx, u0, w, "box", bc, T, engine="direct", fuse_steps=tf)
+            assert rel(got, oracle.run(u0, w, bc, T)) <= TOL, (ndim, r, tf, bc, generic)
+    # star (Heat-3D) exercises the single-column planes
+    w = synth.random_weights("heat3d")
+    u0 = synth.grid((45, 70, 99), seed=62)
+    for bc in ("fixed", "periodic"):
+        got, _ = run_gpu(csx, u0, w, "star", bc, 4, engine="direct")
+        assert rel(got, oracle.run(u0, w, bc, 4)) <= TOL, ("heat3d", bc, generic)
+
+
 @pytest.mark.parametrize("pad,dirty", [(0, 0), (1, 0), (0, 1), (1, 1), (2, 1), (3, 1)])
 @pytest.mark.parametrize("bc", ["fixed", "periodic"])
 def test_s2r_breakdown_variants(csx, pad, dirty, bc):
