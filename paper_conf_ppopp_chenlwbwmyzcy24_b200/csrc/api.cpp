@@ -596,25 +596,46 @@ csx_status run_local(csx_plan_s* p, const double* d_in, double* d_out, int64_t T
   const int real[3] = {p->ndim == 3, p->ndim >= 2, 1};
   View b[2];
   for (int i = 0; i < 2; ++i) b[i] = View{p->d_buf[i] + pd.origin(), pd.s0, pd.s1};
-  cudaError_t e = launch_pack(d_in, b[0], p->E, st);
-  if (e != cudaSuccess) return cuda_fail(e, "pack");
-  p->n_launches += 1;
+  const int64_t nmain = T / p->tf;
+  const int rem = (int)(T % p->tf);
+  const int64_t npass = nmain + (rem ? 1 : 0);
+  // Pass depths (reading A8): nmain passes of Tf then the remainder.  A remainder of 1 after at
+  // least one full pass of Tf >= 3 is folded with the last full pass into two passes of
+  // ceil/floor((Tf+1)/2) — same pass count, and on the DMMA-bound 2D path two nk = 5 passes cost
+  // less than nk = 7 + nk = 3 (12 + 12 vs 20 + 6 DMMAs per 64 outputs, the nk = 3 pass being
+  // HBM-bound at its full sweep).  Kept when CSX_FOLD_REMAINDER=0.
+  const char* fr = getenv("CSX_FOLD_REMAINDER");
+  const bool fold = rem == 1 && nmain >= 1 && p->tf >= 3 && p->ndim >= 2 && !(fr && fr[0] == '0');
+  auto depth = [&](int64_t i) -> int {
+    if (fold && i >= nmain - 1) return i == nmain - 1 ? (p->tf + 2) / 2 : (p->tf + 1) / 2;
+    return i < nmain ? p->tf : rem;
+  };
+  // FIXED TC_TILE 2D / 3D: the first pass stages its tiles straight from the user's dense d_in
+  // through a TMA tensor map (out-of-grid halo boxes zero-filled; only held frame points and
+  // the k_band-recomputed band see them), so no pack into the padded layout.  Not in place for a
+  // single pass (its tiles would read halos other tiles already overwrote).
+  const bool dense_src = p->engine == CSX_ENGINE_TC_TILE && p->ndim >= 2 && p->bc == CSX_BC_FIXED &&
+                         (d_in != d_out || npass > 1) && tile_reads_dense(d_in, p->E[2]);
+  cudaError_t e = cudaSuccess;
+  if (!dense_src) {
+    e = launch_pack(d_in, b[0], p->E, st);
+    if (e != cudaSuccess) return cuda_fail(e, "pack");
+    p->n_launches += 1;
+  }
   const int nghost = real[0] + real[1] + real[2];
   if (p->bc == CSX_BC_PERIODIC) {
     e = launch_ghost_fill(b[0], p->E, real, real, p->halo, st);
     if (e != cudaSuccess) return cuda_fail(e, "ghost fill");
     p->n_launches += nghost;
   }
-  const int64_t nmain = T / p->tf;
-  const int rem = (int)(T % p->tf);
-  const int64_t npass = nmain + (rem ? 1 : 0);
   const View out{d_out, p->E[1] * p->E[2], p->E[2]};
   int cur = 0;
   for (int64_t i = 0; i < npass; ++i) {
-    const int tfp = i < nmain ? p->tf : rem;
+    const int tfp = depth(i);
     const bool last = i == npass - 1;
     PassCtx c;
     c.src = CView{b[cur].p, b[cur].s0, b[cur].s1, pd.O[0], pd.O[1], pd.O[2], pd.A[0]};
+    if (i == 0 && dense_src) c.src = CView{d_in, p->E[1] * p->E[2], p->E[2], 0, 0, 0, p->E[0]};
     c.dst = last ? out : b[cur ^ 1];
     for (int a = 0; a < 3; ++a) { c.E[a] = p->E[a]; c.gorg[a] = 0; }
     csx_status s = run_pass(p, p->passes[tfp - 1], c, st);

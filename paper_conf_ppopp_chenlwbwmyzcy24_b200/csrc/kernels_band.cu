@@ -80,7 +80,10 @@ __global__ void __launch_bounds__(256) k_band(BandArgs a) {
       if (s == 1) {
         const double* c = a.src.p + (NDIM == 2 ? y * a.src.s1 : 0) + x;
         if (hold) {
-          v = *c;
+          // a held point outside the GLOBAL grid feeds only held points: its value is never used,
+          // and a dense source (first pass reading the user's grid) has no ghost cell there
+          const bool out = gx < 0 || gx >= a.G2 || (NDIM == 2 && (gy < 0 || gy >= a.G1));
+          v = out ? 0.0 : *c;
         } else {
           v = 0.0;
 #pragma unroll

@@ -19,6 +19,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <type_traits>
 
 #include "csx_run.h"
 #include "kernels.cuh"
@@ -56,7 +57,8 @@ __global__ void __launch_bounds__(128) k_direct1d(DirectArgs a, Direct1DW W) {
     const bool edge = a.fixed_bc && (g0 < R || g0 + V > G - R);
     // one step in -> out: the R neighbours across the lane boundary by shuffles; FIXED edge
     // lanes hold the frame points
-    auto step = [&](const double (&in)[V], double (&out)[V]) {
+    auto step = [&](const double (&in)[V], double (&out)[V], auto edge_c) {
+      constexpr bool EDGE = decltype(edge_c)::value;
       double l[R], r[R];
 #pragma unroll
       for (int k = 0; k < R; ++k) {
@@ -72,20 +74,32 @@ __global__ void __launch_bounds__(128) k_direct1d(DirectArgs a, Direct1DW W) {
           const double v = j < 0 ? l[j + R] : (j >= V ? r[j - V] : in[j]);
           acc = fma(W.w[k], v, acc);
         }
-        const int64_t gi = g0 + i;
-        out[i] = (edge && (gi < R || gi >= G - R)) ? in[i] : acc;
+        if (EDGE) {
+          const int64_t gi = g0 + i;
+          out[i] = (gi < R || gi >= G - R) ? in[i] : acc;
+        } else {
+          out[i] = acc;
+        }
       }
     };
     double y[V];
     int s = 0;
-    for (; s + 1 < a.tf; s += 2) {  // two steps per trip: x -> y -> x, no register copies
-      step(x, y);
-      step(y, x);
-    }
-    if (s < a.tf) {
-      step(x, y);
+    if (edge) {
+      for (; s < a.tf; ++s) {
+        step(x, y, std::true_type{});
 #pragma unroll
-      for (int i = 0; i < V; ++i) x[i] = y[i];
+        for (int i = 0; i < V; ++i) x[i] = y[i];
+      }
+    } else {
+      for (; s + 1 < a.tf; s += 2) {  // two steps per trip: x -> y -> x, no register copies
+        step(x, y, std::false_type{});
+        step(y, x, std::false_type{});
+      }
+      if (s < a.tf) {
+        step(x, y, std::false_type{});
+#pragma unroll
+        for (int i = 0; i < V; ++i) x[i] = y[i];
+      }
     }
 #pragma unroll
     for (int i = 0; i < V; i += 2) {

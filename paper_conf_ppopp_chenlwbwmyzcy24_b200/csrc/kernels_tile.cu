@@ -137,6 +137,24 @@ static bool make_tmap(S2RArgs& a, int bx, int by, CUtensorMap* map) {
   return true;
 }
 
+// Host: can the TC_TILE 2D / 3D kernels stage their tiles straight from a DENSE grid (the user's
+// d_in: no ghost cells, row pitch E2)?  The TMA tensor map zero-fills the halo boxes that fall
+// outside the grid, which only the held FIXED frame and the band recomputed by k_band could see.
+bool tile_reads_dense(const double* p, int64_t E2) {
+  const char* e = getenv("CSX_TMA");
+  if (e && e[0] == '0') return false;
+  const char* d = getenv("CSX_DENSE_SRC");
+  if (d && d[0] == '0') return false;
+  void* fn = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess ||
+      q != cudaDriverEntryPointSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return (reinterpret_cast<uintptr_t>(p) & 15) == 0 && E2 % 2 == 0;
+}
+
 // Programmatic dependent launch (sm_90+): the kernels below are launched with programmatic
 // stream serialisation (launch_pdl), so pass p+1's CTAs are scheduled onto SMs as pass p's CTAs
 // retire.  Everything before pdl_begin() touches only smem and the plan's constant tables;
@@ -888,7 +906,10 @@ static cudaError_t launch_tile_cfg(S2RArgs a, cudaStream_t st) {
   a.ntiles = (int64_t)a.tiles_x * set_ranges(a, a.tiles_y, C::BM, a.E1, C::R);
   if (a.ntiles == 0) return cudaSuccess;
   CUtensorMap tmap;
-  if (!make_tmap(a, C::TP, C::RR, &tmap)) a.use_tma = 0;
+  if (!make_tmap(a, C::TP, C::RR, &tmap)) {
+    if (a.src.o2 == 0) return cudaErrorNotSupported;  // dense source: no ghost cells to overread
+    a.use_tma = 0;
+  }
   cudaError_t e = cudaFuncSetAttribute(k_tile2d<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
   if (e != cudaSuccess) return e;
   int occ = 0;

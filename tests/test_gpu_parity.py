@@ -140,6 +140,28 @@ def test_signed_weights_general_radius(csx):
                 assert rel(got, oracle.run(u0, w, bc, 4)) <= TOL, (ndim, r, bc, engine)
 
 
+@pytest.mark.parametrize("name,ext", [("box2d9p", (130, 200)), ("box2d9p", (131, 201)),
+                                      ("heat2d", (64, 66)), ("box2d49p", (90, 130)),
+                                      ("heat3d", (40, 35, 70)), ("box3d27p", (33, 40, 66))])
+def test_dense_source_first_pass(csx, monkeypatch, name, ext):
+    """FIXED TC_TILE 2D/3D: the first pass stages tiles straight from the user's dense grid
+    (TMA zero-fills the out-of-grid halo; no pack).  Bitwise equal to the packed path
+    (CSX_DENSE_SRC=0), equal to the oracle, in place and out of place, T below / at / above Tf
+    (odd row lengths fall back to the pack)."""
+    s = synth.SHAPES[name]
+    w = synth.random_weights(name)
+    u0 = synth.grid(ext, seed=17)
+    for T in (1, 3, 4, 7):
+        for inplace in (False, True):
+            got, info = run_gpu(csx, u0, w, s.kind, "fixed", T, inplace=inplace)
+            assert info["engine_name"] == "tc_tile"
+            monkeypatch.setenv("CSX_DENSE_SRC", "0")
+            packed, _ = run_gpu(csx, u0, w, s.kind, "fixed", T, inplace=inplace)
+            monkeypatch.delenv("CSX_DENSE_SRC")
+            assert np.array_equal(got, packed), (name, ext, T, inplace)
+            assert rel(got, oracle.run(u0, w, "fixed", T)) <= TOL, (name, ext, T, inplace)
+
+
 def test_edge_cases(csx):
     w = synth.random_weights("box2d9p")
     u0 = synth.grid((40, 72), seed=3)
