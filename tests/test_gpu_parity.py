@@ -227,18 +227,28 @@ def test_full_size_sampled_box2d9p(csx):
     assert got.min() >= u0.min() and got.max() <= u0.max()
 
 
-@pytest.mark.parametrize("name,ext,T", [("box2d49p", (10240, 10240), 100),
-                                        ("box3d27p", (512, 512, 512), 50),
-                                        ("heat3d", (512, 512, 512), 50),
-                                        ("heat1d", (10240000,), 1000)])
-def test_full_size_sampled(csx, name, ext, T):
+@pytest.mark.parametrize("name,ext,T,tf", [("box2d49p", (10240, 10240), 100, 0),
+                                           ("star2d13p", (10240, 10240), 100, 0),
+                                           ("star2d13p", (10240, 10240), 100, 2),
+                                           ("box2d49p", (10240, 10240), 100, 2),
+                                           ("heat2d", (10240, 10240), 100, 0),
+                                           ("box3d27p", (512, 512, 512), 50, 0),
+                                           ("heat3d", (512, 512, 512), 50, 0),
+                                           ("heat1d", (10240000,), 1000, 0),
+                                           ("1d5p", (10240000,), 1000, 0)])
+def test_full_size_sampled(csx, name, ext, T, tf):
+    """Every BASELINE config at full size and full T in bench.py's launch configuration (auto
+    engine; C3 also at its "multi-step fused" Tf = 2): sampled outputs, incl. corners and the
+    FIXED frame / band, against the oracle's dependence cones."""
     s = synth.SHAPES[name]
     w = synth.random_weights(name)
     u0 = synth.grid(ext)
-    got, info = run_gpu(csx, u0, w, s.kind, "fixed", T)
+    got, info = run_gpu(csx, u0, w, s.kind, "fixed", T, fuse_steps=tf)
     rng = np.random.default_rng(1)
     pts = [tuple(int(rng.integers(0, e)) for e in ext) for _ in range(6)]
-    pts += [tuple(0 for _ in ext), tuple(e - 1 for e in ext), tuple(s.radius for _ in ext)]
+    band = s.radius * info["fuse_steps"]
+    pts += [tuple(0 for _ in ext), tuple(e - 1 for e in ext), tuple(s.radius for _ in ext),
+            tuple(band - 1 for _ in ext), tuple(e - band for e in ext)]
     ref = oracle.sample(u0, w, "fixed", T, pts)
     vals = np.array([got[p] for p in pts])
     assert np.max(np.abs(vals - ref)) / np.max(np.abs(got)) <= TOL, info
