@@ -162,6 +162,25 @@ class ClockSampler:
                 "timed_region_s": round(t1 - t0, 4), "period_ms": self.period}
 
 
+# The JSON line is the only thing bench.py may put on stdout; NCCL's init banner ("NCCL version
+# ...", printed on stdout by every communicator init, ours and torch's) and any other library
+# chatter are sent to stderr by pointing fd 1 there for the run.
+_JSON_OUT = None
+
+
+def emit(line):
+    out = _JSON_OUT if _JSON_OUT is not None else sys.stdout
+    print(json.dumps(line), file=out, flush=True)
+
+
+def quiet_stdout():
+    global _JSON_OUT
+    if _JSON_OUT is None:
+        sys.stdout.flush()
+        _JSON_OUT = os.fdopen(os.dup(1), "w")
+        os.dup2(2, 1)
+
+
 def algorithmic_mma(ndim, nk, engine, points, tc_planes):
     """DMMA.8x8x4 per pass over `points` outputs: Eq 13 generalised by
     reading A7 (N fragments) and 3D planes for TC_S2R; 4x2/2x4 blocks for TC_TILE 2D/3D and
@@ -239,7 +258,7 @@ def run_reference(args, cfg_name):
             "cpu_baseline": {"kind": "oracle", "cores": cores, "sample": sample, "value": value,
                              "unit": UNIT},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-    print(json.dumps(line), flush=True)
+    emit(line)
 
 
 def main():
@@ -270,6 +289,7 @@ def main():
     ap.add_argument("--prof-every", type=int, default=8,
                     help="time every n-th dominant-kernel launch with CUDA events (0: none)")
     args = ap.parse_args()
+    quiet_stdout()
     if args.warmup < 3:
         args.warmup = 3  # timing rule: W >= 3
 
@@ -535,7 +555,7 @@ def main():
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_oracle_sample(shape, gext, T, bc, w)
     if rank == 0:
-        print(json.dumps(line), flush=True)
+        emit(line)
     if comm is not None:
         csx.csx_comm_destroy(comm)
     plan.close()
