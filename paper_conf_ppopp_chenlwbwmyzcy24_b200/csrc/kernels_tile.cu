@@ -466,10 +466,14 @@ static int tile_variant() {
 // DMMA warps compute output plane zo from the NK staged planes zo-R .. zo+R (every tensor-core z
 // offset is a K-slice group of the same GEMM; single-tap z offsets — the star arms, reading A9 —
 // are DFMAs on the same staged planes), then release plane zo-R, which no later output needs.
-template <int NK_, int G_, int WM_, int WN_, int STAGES_, int ZCH_, int CG_ = 1>
+template <int NK_, int G_, int WM_, int WN_, int STAGES_, int ZCH_, int CG_ = 1, int KO_ = 0>
 struct Tile3DCfg {
   static constexpr int NK = NK_, A = 4, B = 2, KC = 4 * ((2 + NK - 1 + 3) / 4), G = G_, WM = WM_,
                        WN = WN_, STAGES = STAGES_, ZCH = ZCH_, CG = CG_;
+  // DMMA issue order inside a TC plane: 0 = by input row (an A fragment feeds every block whose
+  // window holds the row; consecutive DMMAs often hit the same accumulator chain), 1 = k-slice
+  // outer, blocks inner (G independent chains between dependent DMMAs; one LDS per DMMA)
+  static constexpr int KO = KO_;
   static constexpr int R = (NK - 1) / 2;
   static constexpr int ODD = R & 1;  // staged col = region col + ODD (16-B aligned rows)
   static constexpr int KR = A + NK - 1;
@@ -590,7 +594,20 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
 #pragma unroll
       for (int dz = 0; dz < C::NK; ++dz) {
         const double* stg = smem + slot[dz] * C::STAGE_A;
-        if (tc_mask & (1 << dz)) {
+        if ((tc_mask & (1 << dz)) && C::KO == 1) {
+          const double* base = stg + lane_off;
+#pragma unroll
+          for (int rho = 0; rho < C::KR; ++rho)
+#pragma unroll
+            for (int h = 0; h < C::KC / 4; ++h)
+#pragma unroll
+              for (int j = 0; j < C::G; ++j)
+#pragma unroll
+                for (int cg = 0; cg < C::CG; ++cg)
+                  dmma_t(acc[cg][j][0], acc[cg][j][1],
+                         base[(C::A * j + rho) * C::TP + cg * 8 * C::B + 4 * h],
+                         wf[dz][rho * (C::KC / 4) + h]);
+        } else if (tc_mask & (1 << dz)) {
           const double* base = stg + lane_off;
 #pragma unroll
           for (int ra = 0; ra < C::A * C::G + C::NK - 1; ++ra) {
@@ -681,6 +698,8 @@ using Tile3D3 = Tile3DCfg<3, 8, 2, 2, 5, 32>;      // CTA 64 x 32 outputs, 4 DMM
 using Tile3D3b = Tile3DCfg<3, 4, 4, 1, 5, 32, 2>;  // CTA 64 x 32, 4 warps of 4 block rows x 2 column groups
 using Tile3D3c = Tile3DCfg<3, 8, 2, 4, 6, 32>;     // CTA 64 x 64 outputs, 8 DMMA warps, 6-plane ring
 using Tile3D3d = Tile3DCfg<3, 2, 8, 1, 5, 32, 2>;  // CTA 64 x 32, 8 warps of 2 block rows x 2 column groups
+using Tile3D3k = Tile3DCfg<3, 8, 2, 2, 5, 32, 1, 1>;  // Tile3D3, k-slice-outer DMMA order
+using Tile3D3ck = Tile3DCfg<3, 8, 2, 4, 6, 32, 1, 1>;  // Tile3D3c, k-slice-outer DMMA order
 
 
 // ------------------------------------------------------------------------------------------
@@ -949,10 +968,13 @@ cudaError_t launch_tile(int ndim, int nk, const S2RArgs& a, cudaStream_t st) {
       if (e && e[0] == '2') return launch_tile3d_cfg<Tile3D3c>(a, a.tc_mask, st);
       if (e && e[0] == '3') return launch_tile3d_cfg<Tile3D3d>(a, a.tc_mask, st);
       if (e && e[0] == '0') return launch_tile3d_cfg<Tile3D3>(a, a.tc_mask, st);
+      if (e && e[0] == '8') return launch_tile3d_cfg<Tile3D3k>(a, a.tc_mask, st);
+      if (e && e[0] == '9') return launch_tile3d_cfg<Tile3D3ck>(a, a.tc_mask, st);
       // default: star shapes (one TC plane, HBM-bound) take the 64 x 64 tile with 8 DMMA warps
       // (less halo per plane); box shapes (DMMA-bound) the 64 x 32 tile at 2 CTAs / SM
       // (measured)
-      if (__builtin_popcount((unsigned)a.tc_mask) <= 1) return launch_tile3d_cfg<Tile3D3c>(a, a.tc_mask, st);
+      // (k-slice-outer DMMA order: 287 vs 283 GSt/s on Heat-3D, but 184 vs 196 on Box-3D27P)
+      if (__builtin_popcount((unsigned)a.tc_mask) <= 1) return launch_tile3d_cfg<Tile3D3ck>(a, a.tc_mask, st);
       return launch_tile3d_cfg<Tile3D3>(a, a.tc_mask, st);
     }
     return cudaErrorNotSupported;

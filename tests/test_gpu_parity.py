@@ -254,6 +254,20 @@ def test_full_size_sampled(csx, name, ext, T, tf):
     assert np.max(np.abs(vals - ref)) / np.max(np.abs(got)) <= TOL, info
 
 
+@pytest.mark.parametrize("variant", ["0", "1", "2", "3", "8", "9"])
+def test_parity_3d_tile_variants(csx, monkeypatch, variant):
+    """Every TC_TILE 3D CTA geometry / DMMA order (CSX_TILE3D_VARIANT), star and box, ragged
+    (y, x) tiles and z chunks, both boundaries."""
+    monkeypatch.setenv("CSX_TILE3D_VARIANT", variant)
+    for name, ext in (("heat3d", (70, 37, 45)), ("box3d27p", (9, 70, 150)), ("box3d27p", (37, 5, 9))):
+        s = synth.SHAPES[name]
+        u0 = synth.grid(ext, seed=33)
+        w = synth.random_weights(name)
+        for bc in ("fixed", "periodic"):
+            got, info = run_gpu(csx, u0, w, s.kind, bc, 3, engine="tc_tile")
+            assert rel(got, oracle.run(u0, w, bc, 3)) <= TOL, (name, ext, bc, variant)
+
+
 @pytest.mark.parametrize("name", ["heat3d", "box3d27p"])
 @pytest.mark.parametrize("engine", ["tc_tile", "tc_s2r"])
 def test_parity_3d_zchunks(csx, name, engine):
