@@ -283,6 +283,9 @@ def main():
                     help="multi-GPU decomposition: slabs along the slowest axis (default) or a "
                          "p0 x p1 pencil / block grid over the two slowest axes (NCCL exchange; "
                          "--gpus 1 runs the 1 x 1 pencil path)")
+    ap.add_argument("--no-graph", dest="graph", action="store_false",
+                    help="single GPU: launch every pass eagerly instead of replaying the step's "
+                         "pass sequence as one CUDA graph (csx_plan_set_graph, the default)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-comparator", action="store_true")
@@ -412,7 +415,15 @@ def main():
     barrier_sync()
     # the dominant kernel's duration is sampled live: every --prof-every-th main-pass launch is
     # bracketed by CUDA events on its stream (events between kernels break PDL chaining)
-    csx.csx_profile_enable(plan.handle, args.prof_every)
+    graph = args.graph and world == 1 and not pencil
+    if graph:  # the pass sequence is captured by the warm-up steps and replayed in the timed ones
+        plan.set_graph(True)
+        for _ in range(2):
+            step()
+        barrier_sync()
+    # (graph replay carries no per-kernel events: the dominant kernel is then timed in one extra
+    # eager step after the timed region)
+    csx.csx_profile_enable(plan.handle, 0 if graph else args.prof_every)
     csx.csx_profile_read(plan.handle, reset=True)
     # Timing rule: grids larger than L2 (126 MB) need no flush; smaller ones get a 256 MB write
     # between timed steps, outside the per-step CUDA-event windows.
@@ -434,6 +445,14 @@ def main():
         clk.mark("end")
     ms_total = sum(e0.elapsed_time(e1) for e0, e1 in evs)
     tc_ms, tc_launches, launches = csx.csx_profile_read(plan.handle, reset=True)
+    tc_scale = 1.0  # steps the profiled launches cover, relative to the timed region
+    if graph and args.prof_every > 0:
+        csx.csx_profile_enable(plan.handle, args.prof_every)
+        step()
+        torch.cuda.synchronize()
+        tc_ms, tc_launches, _ = csx.csx_profile_read(plan.handle, reset=True)
+        tc_scale = 1.0 / args.steps
+        plan.set_graph(False)
     csx.csx_profile_enable(plan.handle, False)
     if world > 1:
         t = torch.tensor([ms_total], device=red_dev, dtype=torch.float64)
@@ -476,7 +495,7 @@ def main():
                     "launches": tc_launches,
                     "per_launch": f"16 B x {local_points} points (1 read + 1 write per pass)",
                     "tensor_frac": flops / avg_s / 1e12 / dmma}
-        roof["tc_share_of_step"] = tc_ms / ms_total if ms_total > 0 else None
+        roof["tc_share_of_step"] = tc_ms / (ms_total * tc_scale) if ms_total > 0 else None
         roof["timed_every"] = args.prof_every
 
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -484,7 +503,7 @@ def main():
             "scaling": "weak", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic (splitmix64 seed 20240302, dyadic physical weights)",
             "config": {"workload": args.config, "shape": shape, "grid": list(gext), "T": T, "bc": bc,
-                       "fuse_steps": tfm, "nk": nk, "engine": engine,
+                       "fuse_steps": tfm, "nk": nk, "engine": engine, "cuda_graph": graph,
                        "s2r_variant": args.s2r_variant if engine == "tc_s2r" else None,
                        "parallelism": (f"pencil{p0}x{p1}" if pencil else f"slab{world}" if world > 1 else "single"),
                        "exchange": exchange,

@@ -87,6 +87,14 @@ int csx_auto_fuse_steps(int ndim, int radius, csx_engine engine);
  * this plan's (ndim, radius, Tf). */
 csx_status csx_plan_set_engine(csx_plan_t plan, csx_engine engine);
 
+/* CUDA-graph replay of csx_run (default off).  With on != 0, csx_run captures the pass sequence
+ * of a (d_in, d_out, timesteps) triple into a CUDA graph (after running it eagerly once) and
+ * replays later calls with the same triple as one cudaGraphLaunch on the caller's stream; a
+ * different triple re-captures.  Same results as eager runs; the plan must not be used on two
+ * streams at once (as for eager runs).  Ignored while csx_profile_enable is active.  Errors:
+ * INVALID_ARGUMENT (NULL plan); capture / instantiate failures surface as CUDA from csx_run. */
+csx_status csx_plan_set_graph(csx_plan_t plan, int on);
+
 /* TC_S2R breakdown variants (Fig 6, P.1865-1950), 2D only: padding = 0 uses the bare
  * stencil2row pitch nk*rr (Fig 5's conflicting 266) instead of the conflict-free one (268);
  * dirty_bits = 0 replaces the dirty-bits padding by conditional stores in the LUT copy loop.

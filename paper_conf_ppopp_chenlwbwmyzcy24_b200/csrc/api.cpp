@@ -35,6 +35,15 @@ csx_status cuda_fail(cudaError_t e, const char* where) {
     if (e_ != cudaSuccess) return cuda_fail(e_, where); \
   } while (0)
 
+// drop a captured csx_run graph (engine / variant changes make it stale)
+static void graph_reset(csx_plan_s* p) {
+  if (p->g_exec) {
+    cudaGraphExecDestroy((cudaGraphExec_t)p->g_exec);
+    p->g_exec = nullptr;
+  }
+  p->g_T = -1;
+}
+
 // Tile shape of the direct kernel (engine DIRECT and the FIXED band fix-up).
 void direct_tile(int ndim, int* B) {
   if (ndim == 1) { B[0] = 1; B[1] = 1; B[2] = 1024; }
@@ -213,6 +222,8 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
         if (need > p->s2r_elems) {
           cudaFree(p->d_s2r);
     cudaFree(p->d_pstage);
+    if (p->g_exec) cudaGraphExecDestroy((cudaGraphExec_t)p->g_exec);
+    if (p->g_stream) cudaStreamDestroy((cudaStream_t)p->g_stream);
     if (p->peer) {
       csx_peer_s* q = p->peer;
       for (void* ptr : q->opened) cudaIpcCloseMemHandle(ptr);
@@ -376,6 +387,7 @@ int csx_auto_fuse_steps(int ndim, int radius, csx_engine engine) {
 }
 
 csx_status csx_plan_set_s2r_variant(csx_plan_t p, int padding, int dirty_bits) {
+  if (p) graph_reset(p);
   if (!p) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL plan");
   // padding = 2: breakdown variant II (padding + dirty bits, tessellation on CUDA cores);
   // padding = 3: breakdown variant I (explicit stencil2row in HBM, CUDA-core tessellation)
@@ -407,6 +419,7 @@ csx_status csx_plan_set_s2r_variant(csx_plan_t p, int padding, int dirty_bits) {
 }
 
 csx_status csx_plan_set_engine(csx_plan_t p, csx_engine e) {
+  if (p) graph_reset(p);
   if (!p) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL plan");
   if (e == CSX_ENGINE_AUTO) {
     p->engine_req = e;
@@ -441,7 +454,59 @@ csx_status csx_run(csx_plan_t p, const double* d_in, double* d_out, int64_t T, v
   }
   s = ensure_grid(p, &p->pad, p->d_buf, p->E);
   if (s != CSX_OK) return s;
-  return run_local(p, d_in, d_out, T, st);
+  if (!p->graph_on || p->prof > 0) return run_local(p, d_in, d_out, T, st);
+  // Graph mode: replay the captured pass sequence if (d_in, d_out, T) match; otherwise run
+  // eagerly (first use: lazy allocations, tensor maps) and capture the same sequence on the
+  // plan's non-blocking stream for the next call.  The replay is one cudaGraphLaunch on the
+  // caller's stream (the legacy default stream included); PDL edges are kept in the graph.
+  if (p->g_exec && p->g_in == d_in && p->g_out == d_out && p->g_T == T) {
+    CSX_CUDA(cudaGraphLaunch((cudaGraphExec_t)p->g_exec, st), "cudaGraphLaunch");
+    p->n_launches += p->g_launches;
+    p->n_tc_launches += p->g_tc_launches;
+    return CSX_OK;
+  }
+  s = run_local(p, d_in, d_out, T, st);
+  if (s != CSX_OK) return s;
+  if (p->g_exec) {
+    cudaGraphExecDestroy((cudaGraphExec_t)p->g_exec);
+    p->g_exec = nullptr;
+  }
+  if (!p->g_stream) {
+    cudaStream_t cs;
+    CSX_CUDA(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking), "capture stream");
+    p->g_stream = cs;
+  }
+  cudaStream_t cs = (cudaStream_t)p->g_stream;
+  const int64_t l0 = p->n_launches, t0 = p->n_tc_launches;
+  CSX_CUDA(cudaStreamBeginCapture(cs, cudaStreamCaptureModeRelaxed), "begin capture");
+  s = run_local(p, d_in, d_out, T, cs);
+  cudaGraph_t g = nullptr;
+  const cudaError_t ec = cudaStreamEndCapture(cs, &g);
+  if (s != CSX_OK) {
+    if (g) cudaGraphDestroy(g);
+    return s;
+  }
+  if (ec != cudaSuccess) return cuda_fail(ec, "end capture");
+  cudaGraphExec_t ge = nullptr;
+  const cudaError_t ei = cudaGraphInstantiate(&ge, g, 0);
+  cudaGraphDestroy(g);
+  if (ei != cudaSuccess) return cuda_fail(ei, "cudaGraphInstantiate");
+  p->g_exec = ge;
+  p->g_in = d_in;
+  p->g_out = d_out;
+  p->g_T = T;
+  p->g_launches = p->n_launches - l0;  // capture counted the launches without running them
+  p->g_tc_launches = p->n_tc_launches - t0;
+  p->n_launches = l0;
+  p->n_tc_launches = t0;
+  return CSX_OK;
+}
+
+csx_status csx_plan_set_graph(csx_plan_t p, int on) {
+  if (!p) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL plan");
+  p->graph_on = on != 0;
+  graph_reset(p);
+  return CSX_OK;
 }
 
 csx_status csx_run_host(csx_plan_t p, const double* h_in, double* h_out, int64_t T, void* stream) {
@@ -519,6 +584,8 @@ csx_status csx_plan_destroy(csx_plan_t p) {
     }
     cudaFree(p->d_s2r);
     cudaFree(p->d_pstage);
+    if (p->g_exec) cudaGraphExecDestroy((cudaGraphExec_t)p->g_exec);
+    if (p->g_stream) cudaStreamDestroy((cudaStream_t)p->g_stream);
 
     cudaSetDevice(cur);
   }

@@ -143,6 +143,14 @@ struct csx_plan_s {
   void* side = nullptr;            // cudaStream_t
   void* ev_fork = nullptr;         // cudaEvent_t
   void* ev_join = nullptr;
+  // CUDA graph replay of csx_run (csx_plan_set_graph): the pass sequence of one
+  // (d_in, d_out, T) captured once and replayed with one cudaGraphLaunch
+  int graph_on = 0;
+  void* g_exec = nullptr;          // cudaGraphExec_t
+  void* g_stream = nullptr;        // non-blocking capture stream
+  const double* g_in = nullptr;
+  double* g_out = nullptr;
+  int64_t g_T = -1, g_launches = 0, g_tc_launches = 0;
   // measurement hooks
   int prof = 0;  // 0 off, n: time every n-th main-pass TC launch
   std::vector<void*> prof_events;  // cudaEvent_t pairs around TC launches

@@ -236,9 +236,10 @@ constexpr int s2r_pitch_dev(int min_pitch) {
 
 // Compile-time geometry of one TC_TILE instantiation.
 template <int NK_, int A_, int B_, int KC_, int G_, int WM_, int WN_, int STAGES_, int CG_ = 1,
-          int MINB_ = 1>
+          int MINB_ = 1, int KO_ = 0>
 struct TileCfg {
   static constexpr int NK = NK_, A = A_, B = B_, KC = KC_, G = G_, WM = WM_, WN = WN_;
+  static constexpr int KO = KO_;                    // 1: k-slice-outer DMMA order (Tile3DCfg)
   static constexpr int MINB = MINB_;                // CTAs per SM the registers are sized for
   static constexpr int STAGES = STAGES_;
   static constexpr int CG = CG_;                    // 8-block column groups per warp
@@ -352,19 +353,32 @@ __global__ void __launch_bounds__(C::NT, C::MINB)
     // Stream the warp's input rows; each A fragment (4 cells of one row) feeds every output
     // block whose window contains the row.  Block j is complete after input row A*j + KR - 1 and
     // (interior tiles) is stored right there, so the epilogue interleaves with the DMMA stream.
+    if (C::KO == 1) {
 #pragma unroll
-    for (int ra = 0; ra < C::A * C::G + C::NK - 1; ++ra) {
+      for (int rho = 0; rho < C::KR; ++rho)
+#pragma unroll
+        for (int h = 0; h < C::KC / 4; ++h)
+#pragma unroll
+          for (int j = 0; j < C::G; ++j)
+#pragma unroll
+            for (int cg = 0; cg < C::CG; ++cg)
+              dmma_t(acc[cg][j][0], acc[cg][j][1], base[(C::A * j + rho) * C::TP + cg * 8 * C::B + 4 * h],
+                     wf[rho * (C::KC / 4) + h]);
+    }
+#pragma unroll
+    for (int ra = (C::KO == 1 ? C::KR - 1 : 0); ra < C::A * C::G + C::NK - 1; ++ra) {
       double f[C::CG][C::KC / 4];
 #pragma unroll
       for (int cg = 0; cg < C::CG; ++cg)
 #pragma unroll
-        for (int h = 0; h < C::KC / 4; ++h) f[cg][h] = base[ra * C::TP + cg * 8 * C::B + 4 * h];
+        for (int h = 0; h < C::KC / 4; ++h)
+          if (C::KO == 0) f[cg][h] = base[ra * C::TP + cg * 8 * C::B + 4 * h];
 #pragma unroll
       for (int h = 0; h < C::KC / 4; ++h)
 #pragma unroll
         for (int j = 0; j < C::G; ++j) {
           const int rho = ra - C::A * j;
-          if (rho >= 0 && rho < C::KR)
+          if (C::KO == 0 && rho >= 0 && rho < C::KR)
 #pragma unroll
             for (int cg = 0; cg < C::CG; ++cg)
               dmma_t(acc[cg][j][0], acc[cg][j][1], f[cg][h], wf[rho * (C::KC / 4) + h]);
@@ -444,6 +458,7 @@ using Tile5c = TileCfg<5, 2, 4, 8, 4, 12, 1, 3, 2>;
 using Tile7c = TileCfg<7, 4, 2, 8, 4, 6, 2, 3, 2>;
 using Tile7d = TileCfg<7, 4, 2, 8, 8, 2, 3, 3, 1, 2>;  // variant 3: 2 CTAs/SM of 6 DMMA warps (64 x 48)
 using Tile7e = TileCfg<7, 4, 2, 8, 8, 2, 4, 2, 1, 2>;  // variant 4: 2 CTAs/SM of 8 DMMA warps (64 x 64)
+using Tile7k = TileCfg<7, 4, 2, 8, 8, 4, 4, 2, 1, 1, 1>;  // variant 5: Tile7b, k-slice-outer DMMA order
 
 // fused windows beyond the paper's one N fragment (reading A7): 8 DMMA warps, CTA 64 x 64,
 // 3-stage ring; the K/4 weight fragments (30 / 42 / 56) stay in registers
@@ -987,7 +1002,7 @@ cudaError_t launch_tile(int ndim, int nk, const S2RArgs& a, cudaStream_t st) {
     case 9: return launch_tile_cfg<Tile9>(a, st);
     case 11: return launch_tile_cfg<Tile11>(a, st);
     case 13: return launch_tile_cfg<Tile13>(a, st);
-    case 7: return v == 4 ? launch_tile_cfg<Tile7e>(a, st) : v == 3 ? launch_tile_cfg<Tile7d>(a, st) : v == 2 ? launch_tile_cfg<Tile7c>(a, st) : v ? launch_tile_cfg<Tile7b>(a, st) : launch_tile_cfg<Tile7>(a, st);
+    case 7: return v == 5 ? launch_tile_cfg<Tile7k>(a, st) : v == 4 ? launch_tile_cfg<Tile7e>(a, st) : v == 3 ? launch_tile_cfg<Tile7d>(a, st) : v == 2 ? launch_tile_cfg<Tile7c>(a, st) : v ? launch_tile_cfg<Tile7b>(a, st) : launch_tile_cfg<Tile7>(a, st);
   }
   return cudaErrorNotSupported;
 }

@@ -383,3 +383,34 @@ def test_sharded_pencil_single_rank(csx, name, ext, T, bc):
     ref = oracle.run(u0, w, bc, T)
     assert rel(got, ref) <= TOL, (name, bc)
     assert rel(got_slab, ref) <= TOL, (name, bc)
+
+
+@pytest.mark.parametrize("name,ext,T", [("box2d9p", (300, 260), 10), ("heat1d", (50000,), 40),
+                                        ("box3d27p", (40, 50, 70), 3), ("heat1d", (1024,), 16)])
+def test_graph_replay(csx, name, ext, T):
+    """csx_plan_set_graph: the first call runs eagerly and captures, later calls with the same
+    (d_in, d_out, T) replay the CUDA graph; a new triple re-captures.  Bitwise equal to eager
+    runs and equal to the oracle (C1 = Heat-1D N=1024, T=16 is the last case)."""
+    s = synth.SHAPES[name]
+    w = synth.random_weights(name)
+    u0 = synth.grid(ext, seed=71)
+    ref = oracle.run(u0, w, "fixed", T)
+    p = csx.Plan(u0.shape, w, shape=s.kind, bc="fixed")
+    d_in = torch.from_numpy(u0).cuda()
+    eager = torch.empty_like(d_in)
+    p.run(d_in, eager, T)
+    p.set_graph(True)
+    outs = [torch.full_like(d_in, -1.0) for _ in range(2)]
+    for k in range(3):                       # capture, replay, replay
+        outs[0].fill_(-1.0)
+        p.run(d_in, outs[0], T)
+        torch.cuda.synchronize()
+        assert torch.equal(outs[0], eager), k
+    p.run(d_in, outs[1], T)                  # new output pointer -> re-capture
+    p.run(d_in, outs[1], T - 1)              # new T -> re-capture
+    torch.cuda.synchronize()
+    p.set_graph(False)
+    p.close()
+    assert torch.equal(outs[1], outs[1])
+    assert rel(outs[0].cpu().numpy(), ref) <= TOL
+    assert rel(outs[1].cpu().numpy(), oracle.run(u0, w, "fixed", T - 1)) <= TOL
