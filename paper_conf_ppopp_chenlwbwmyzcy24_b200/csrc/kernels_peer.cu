@@ -28,9 +28,22 @@ __device__ __forceinline__ void st_release_sys(unsigned long long* p, unsigned l
   asm volatile("st.release.sys.global.u64 [%0], %1;\n" ::"l"(p), "l"(v) : "memory");
 }
 
+__device__ __forceinline__ unsigned long long global_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+// Spin on a peer-written epoch.  A neighbour that never arrives (a rank died or called with a
+// different T) must not hang the GPU: after 60 s the kernel traps, so the run fails with a CUDA
+// error at the caller's next synchronisation instead of spinning forever.
 __device__ __forceinline__ void spin_until(const unsigned long long* p, unsigned long long v) {
   if (!p) return;
-  while (ld_acquire_sys(p) < v) __nanosleep(256);
+  const unsigned long long t0 = global_ns();
+  while (ld_acquire_sys(p) < v) {
+    __nanosleep(256);
+    if (global_ns() - t0 > 60ull * 1000000000ull) __trap();
+  }
 }
 
 __global__ void k_peer_push(PeerPushArgs a) {
