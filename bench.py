@@ -192,6 +192,10 @@ def algorithmic_mma(ndim, nk, engine, points, tc_planes):
         nf = (sw + 7) // 8
         k = nk if ndim == 1 else nk * nk
         return points / (8 * sw) * 2 * math.ceil(k / 4) * nf * tc_planes
+    if engine == "tc_tile" and ndim == 3 and nk == 5:
+        # 3D Tf = 2 by temporal blocking (k_tile3d_tb): two steps of the base stencil (nk = 3,
+        # 4x2 blocks, 6 DMMAs per 64 outputs per TC plane); the recomputed halo is overhead
+        return 2 * points / 64 * 6 * tc_planes
     if engine == "tc_tile":
         # the block shape of smaller K (planner.cpp): 2x4 for nk = 5, 9, 13; 4x2 otherwise
         kdim = lambda a, b: (a + nk - 1) * 4 * math.ceil((b + nk - 1) / 4)

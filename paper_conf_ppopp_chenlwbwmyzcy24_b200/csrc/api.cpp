@@ -173,10 +173,14 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
     a.lut = reinterpret_cast<const int2*>(ps.d_lut);
     a.wc = ps.d_wc;
     if (eng == CSX_ENGINE_TC_TILE) {
-      a.frags = ps.d_tile_frags;
+      // 3D Tf = 2 runs the BASE stencil twice in shared memory (k_tile3d_tb): base fragments,
+      // base weights and the base plane split
+      const Pass& pw = (p->ndim == 3 && ps.tf == 2) ? p->passes[0] : ps;
+      a.frags = pw.d_tile_frags;
+      a.wc = pw.d_wc;
       a.pdl = !band_side && c.part == 0;  // no PDL across the band join / halo-exchange waits
       if (p->ndim == 3)
-        for (int dz = 0; dz < ps.nk; ++dz) a.tc_mask |= ps.plane_is_tc[dz] << dz;
+        for (int dz = 0; dz < pw.nk; ++dz) a.tc_mask |= pw.plane_is_tc[dz] << dz;
       if (p->bc == CSX_BC_FIXED && p->ndim == 1) {  // 1D band recomputed in-kernel
         a.fix_band = p->radius * ps.tf;
         a.r = p->radius;
@@ -188,7 +192,7 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
         // 2D: the edge CTAs leave the band to k_band (Tf > 1) or write the held frame (Tf = 1);
         // 3D (Tf = 1): the frame is written from the staged plane
         a.fix_band = p->radius * ps.tf;
-        a.hold_frame = ps.tf == 1;
+        a.hold_frame = ps.tf == 1 || p->ndim == 3;  // 3D Tf = 2 holds the frame at both levels
         a.r = p->radius;
         a.wbase = p->d_wbase;
         a.gorg0 = c.gorg[0];
@@ -286,7 +290,8 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
     if (e != cudaSuccess) return cuda_fail(e, "direct launch");
     p->n_launches += 1;
   } else if (p->bc == CSX_BC_FIXED && !(eng == CSX_ENGINE_TC_TILE && p->ndim == 1) &&
-             !(eng == CSX_ENGINE_TC_TILE && p->ndim >= 2 && ps.tf == 1)) {  // else done in-kernel
+             !(eng == CSX_ENGINE_TC_TILE && p->ndim >= 2 && ps.tf == 1) &&
+             !(eng == CSX_ENGINE_TC_TILE && p->ndim == 3)) {  // else done in-kernel
     if (ps.tf == 1 || p->ndim == 3) {
       // the composed window is the plain stencil: only the held frame needs restoring
       e = launch_frame_copy(c.src, c.dst, c.E, c.gorg, p->E, real, p->radius, st);

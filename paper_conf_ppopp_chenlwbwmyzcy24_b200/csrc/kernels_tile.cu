@@ -709,6 +709,238 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
   }
 }
 
+// ------------------------------------------------------------------------------------------
+// 3D, two fused time steps by temporal blocking in shared memory (Tf = 2, base radius 1).
+// Composing W twice (the 2D path's kernel fusion, P.1466-1482) would turn the single-tap z arms
+// of a star stencil into 5-tap planes that need the tensor cores (3 TC planes of nk = 5: 3x the
+// DMMAs of Tf = 1 per step).  Instead each pass streams the input planes once and runs the BASE
+// stencil twice: level 1 computes step-1 planes on the tile grown by one cell (its own GEMM
+// tiling, 36 x 80 for a 32 x 64 output tile) into a 3-plane shared-memory ring, level 2 computes
+// the outputs from that ring — the same per-plane GEMM (4x2 output blocks on DMMA.8x8x4,
+// single-tap planes as DFMA) at both levels.  HBM traffic per step halves; DMMAs per step grow
+// by the recomputed halo (~1.2x).  FIXED: both levels hold the frame, so no band fix-up.
+struct Tile3DTB {
+  static constexpr int NK = 3, R = 1, A = 4, B = 2, KC = 4, KR = 6, KS = 6;
+  static constexpr int WM = 2, WN = 4, NCW = 8, NT = 32 * (NCW + 1);
+  static constexpr int G2 = 4;                  // level-2 blocks per warp (column)
+  static constexpr int BM = WM * A * G2;        // 32 output rows
+  static constexpr int BN = WN * 8 * B;         // 64 output cols
+  static constexpr int G1 = 3;                  // level-1 blocks per unit
+  static constexpr int U1R = 3, U1C = 5;        // level-1 units: 3 block-row groups x 5 col groups
+  static constexpr int BM1 = U1R * A * G1;      // 36 >= BM + 2 step-1 rows
+  static constexpr int BN1 = U1C * 8 * B;       // 80 >= BN + 3 step-1 cols
+  static constexpr int TP = 84;                 // plane pitch (input and step-1), even
+  static constexpr int RIN = BM1 + 2;           // staged input rows (38)
+  static constexpr int SIN = RIN * TP;          // doubles per input plane
+  static constexpr int SIN_A = (SIN + 15) / 16 * 16;
+  static constexpr int SL1 = BM1 * TP;          // doubles per step-1 plane
+  static constexpr int SL1_A = (SL1 + 15) / 16 * 16;
+  static constexpr int STAGES = 5;              // input ring
+  static constexpr int ZCH = 32;
+  static constexpr int H = 2;                   // halo of the pass (R * Tf)
+  static constexpr int SMEM = (STAGES * SIN_A + 3 * SL1_A) * 8 + 128;
+  static_assert(TP >= 8 * B * U1C + 4 && TP <= 256 && RIN <= 256, "plane geometry");
+};
+
+// One z-window GEMM of G output blocks (4 x 2 each) for a warp: out rows r0 + 4j + alpha, cols
+// c0 + 2g + beta (+e) of the destination grid whose staged planes `pl[dz]` hold its inputs at
+// (row + dy, col + 1 + dx) (level 1: input planes; level 2: step-1 planes).  TC planes on DMMA,
+// single-tap planes (star z arms) as DFMA on the centre cell.
+template <int G>
+__device__ __forceinline__ void tb_window(double (&acc)[G][2], const double* const (&pl)[3], int r0, int c0,
+                                          int tc_mask, const double (&wf)[3][Tile3DTB::KS],
+                                          const double (&wz)[3], int lane) {
+  using C = Tile3DTB;
+  const int g = lane >> 2, t = lane & 3;
+  const int alpha = (2 * t) / C::B, beta = (2 * t) % C::B;
+#pragma unroll
+  for (int j = 0; j < G; ++j) acc[j][0] = acc[j][1] = 0.0;
+#pragma unroll
+  for (int dz = 0; dz < 3; ++dz) {
+    if (tc_mask & (1 << dz)) {
+      const double* base = pl[dz] + r0 * C::TP + c0 + 1 + C::B * g + t;
+#pragma unroll
+      for (int rho = 0; rho < C::KR; ++rho)
+#pragma unroll
+        for (int j = 0; j < G; ++j)
+          dmma_t(acc[j][0], acc[j][1], base[(C::A * j + rho) * C::TP], wf[dz][rho]);
+    } else if (wz[dz] != 0.0) {
+#pragma unroll
+      for (int j = 0; j < G; ++j) {
+        const double2 v = *reinterpret_cast<const double2*>(
+            pl[dz] + (r0 + C::A * j + alpha + C::R) * C::TP + c0 + C::B * g + beta + C::R + 1);
+        acc[j][0] = fma(wz[dz], v.x, acc[j][0]);
+        acc[j][1] = fma(wz[dz], v.y, acc[j][1]);
+      }
+    }
+  }
+}
+
+__global__ void __launch_bounds__(Tile3DTB::NT, 1)
+    k_tile3d_tb(S2RArgs a, int tc_mask, const __grid_constant__ CUtensorMap tmap) {
+  using C = Tile3DTB;
+  extern __shared__ __align__(128) double smem_raw[];
+  double* smem = ring_base(smem_raw);
+  double* l1 = smem + C::STAGES * C::SIN_A;  // 3 step-1 planes
+  __shared__ __align__(8) uint64_t full[C::STAGES], empty[C::STAGES];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  if (tid == 0) {
+    for (int s = 0; s < C::STAGES; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], C::NCW);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  __syncthreads();
+  pdl_begin();
+  const int ncol = a.tiles_x * a.tiles_y;
+  if (warp == C::NCW) {  // producer: input planes z0-2 .. z1+1 of every work item
+    if (lane == 0) tma_prefetch_desc(&tmap);
+    int q = 0;
+    for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
+      const int zcl = (int)(item / ncol), tile = (int)(item - (int64_t)zcl * ncol);
+      const int64_t zc = slab_map(a, zcl);
+      const int ty = tile / a.tiles_x, tx = tile - ty * a.tiles_x;
+      const int64_t z0 = zc * C::ZCH, z1 = min(a.E0, z0 + C::ZCH);
+      for (int64_t zi = z0 - C::H; zi < z1 + C::H; ++zi, ++q) {
+        const int s = q % C::STAGES, n = q / C::STAGES;
+        if (n > 0) mbar_wait(&empty[s], (uint32_t)((n - 1) & 1));
+        if (lane == 0) {
+          mbar_expect_tx(&full[s], (uint32_t)(C::SIN * 8));
+          tma_load_3d(smem + s * C::SIN_A, &tmap, &full[s], (int)(a.tma_x0 + (int64_t)tx * C::BN - 4),
+                      (int)(a.tma_y0 + (int64_t)ty * C::BM - 2), (int)(a.tma_z0 + zi));
+        }
+      }
+    }
+    return;
+  }
+  double wf[3][C::KS], wz[3];
+#pragma unroll
+  for (int p = 0; p < 3; ++p) {
+#pragma unroll
+    for (int k = 0; k < C::KS; ++k) wf[p][k] = a.frags[(p * C::KS + k) * 32 + lane];
+    wz[p] = a.wc[(p * 3 + 1) * 3 + 1];
+  }
+  const int g = lane >> 2, t = lane & 3;
+  const int alpha = (2 * t) / C::B, beta = (2 * t) % C::B;
+  const bool fixed = a.hold_frame != 0;
+  // level-2 unit of this warp: block rows wm*G2.., column group wn
+  const int wm = warp / C::WN, wn = warp - (warp / C::WN) * C::WN;
+  int q = 0;  // sequence number of the next input plane (producer order)
+  for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
+    const int zcl = (int)(item / ncol), tile = (int)(item - (int64_t)zcl * ncol);
+    const int64_t zc = slab_map(a, zcl);
+    const int ty = tile / a.tiles_x, tx = tile - ty * a.tiles_x;
+    const int64_t z0 = zc * C::ZCH, z1 = min(a.E0, z0 + C::ZCH);
+    const int64_t y0 = (int64_t)ty * C::BM, x0 = (int64_t)tx * C::BN;
+    // global origin of the tile (FIXED holds use global coordinates)
+    const int64_t gy0 = y0 + a.gorg1, gx0 = x0 + a.gorg2;
+    const bool tile_edge = fixed && (gy0 < 2 || gy0 + C::BM + 1 > a.GE1 - 1 || gx0 < 2 ||
+                                     gx0 + C::BN + 1 > a.GE2 - 1);
+    // input planes zl-1, zl, zl+1 for step-1 plane zl: sequence numbers q0 + (zl - (z0-2)) ...
+    const int q0 = q;
+    auto in_plane = [&](int64_t zi) -> const double* {
+      return smem + ((q0 + (int)(zi - (z0 - C::H))) % C::STAGES) * C::SIN_A;
+    };
+    auto wait_in = [&](int64_t zi) {
+      const int qq = q0 + (int)(zi - (z0 - C::H));
+      mbar_wait(&full[qq % C::STAGES], (uint32_t)((qq / C::STAGES) & 1));
+    };
+    auto release_in = [&]() {
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[q % C::STAGES]);
+      ++q;
+    };
+    wait_in(z0 - 2);
+    wait_in(z0 - 1);
+    for (int64_t zl = z0 - 1; zl <= z1; ++zl) {
+      wait_in(zl + 1);
+      // ---- level 1: step-1 plane zl on the grown tile (rows y0-1 .., cols x0-2 ..) ----
+      const double* pin[3] = {in_plane(zl - 1), in_plane(zl), in_plane(zl + 1)};
+      double* dl1 = l1 + (int)((zl - (z0 - 1)) % 3) * C::SL1_A;
+      const int64_t gz1 = zl + a.gorg0;
+      const bool zf1 = fixed && (gz1 < 1 || gz1 >= a.GE0 - 1);
+      for (int u = warp; u < C::U1R * C::U1C; u += C::NCW) {
+        const int ur = u / C::U1C, uc = u - (u / C::U1C) * C::U1C;
+        const int r0 = ur * C::A * C::G1, c0 = uc * 8 * C::B;
+        double acc[C::G1][2];
+        tb_window<C::G1>(acc, pin, r0, c0, tc_mask, wf, wz, lane);
+#pragma unroll
+        for (int j = 0; j < C::G1; ++j) {
+          const int r = r0 + C::A * j + alpha, c = c0 + C::B * g + beta;  // step-1 plane coords
+          double v0 = acc[j][0], v1 = acc[j][1];
+          if (fixed && (zf1 || tile_edge)) {  // held frame points keep the input value
+            const int64_t gy = gy0 - 1 + r, gx = gx0 - 2 + c;
+            const double* ctr = pin[1] + (r + 1) * C::TP + c + 2;
+            const bool yf = zf1 || gy < 1 || gy >= a.GE1 - 1;
+            if (yf || gx < 1 || gx >= a.GE2 - 1) v0 = ctr[0];
+            if (yf || gx + 1 < 1 || gx + 1 >= a.GE2 - 1) v1 = ctr[1];
+          }
+          *reinterpret_cast<double2*>(dl1 + r * C::TP + c) = make_double2(v0, v1);
+        }
+      }
+      release_in();  // input plane zl-1 is not read again
+      asm volatile("bar.sync 1, %0;\n" ::"n"(C::NCW * 32) : "memory");  // step-1 plane zl ready
+      // ---- level 2: output plane zo = zl-1 from step-1 planes zl-2, zl-1, zl ----
+      const int64_t zo = zl - 1;
+      if (zo >= z0) {
+        const double* p1[3] = {l1 + (int)((zl - 2 - (z0 - 1)) % 3) * C::SL1_A,
+                               l1 + (int)((zl - 1 - (z0 - 1)) % 3) * C::SL1_A, dl1};
+        const int r0 = wm * C::A * C::G2, c0 = wn * 8 * C::B;
+        double acc[C::G2][2];
+        tb_window<C::G2>(acc, p1, r0, c0, tc_mask, wf, wz, lane);
+        const int64_t gzo = zo + a.gorg0;
+        const bool zf = fixed && (gzo < 1 || gzo >= a.GE0 - 1);
+        double* plane = a.dst.p + zo * a.dst.s0;
+#pragma unroll
+        for (int j = 0; j < C::G2; ++j) {
+          const int r = r0 + C::A * j + alpha, c = c0 + C::B * g + beta;  // output tile coords
+          const int64_t row = y0 + r, col = x0 + c;
+          if (row >= a.E1 || col >= a.E2) continue;
+          double v0 = acc[j][0], v1 = acc[j][1];
+          if (fixed && (zf || tile_edge)) {
+            const double* ctr = p1[1] + (r + 1) * C::TP + c + 2;
+            const int64_t gy = gy0 + r, gx = gx0 + c;
+            const bool yf = zf || gy < 1 || gy >= a.GE1 - 1;
+            if (yf || gx < 1 || gx >= a.GE2 - 1) v0 = ctr[0];
+            if (yf || gx + 1 < 1 || gx + 1 >= a.GE2 - 1) v1 = ctr[1];
+          }
+          double* p = plane + row * a.dst.s1 + col;
+          if (col + 1 < a.E2 && a.dst_aligned) {
+            *reinterpret_cast<double2*>(p) = make_double2(v0, v1);
+          } else {
+            p[0] = v0;
+            if (col + 1 < a.E2) p[1] = v1;
+          }
+        }
+      }
+      asm volatile("bar.sync 1, %0;\n" ::"n"(C::NCW * 32) : "memory");  // ring slot zl-2 free
+    }
+    release_in();  // input planes z1, z1+1
+    release_in();
+  }
+}
+
+template <class C>
+static cudaError_t launch_tile3d_tb(S2RArgs a, int tc_mask, cudaStream_t st) {
+  a.dst_aligned = ((reinterpret_cast<uintptr_t>(a.dst.p) & 15) == 0) && (a.dst.s1 % 2 == 0) &&
+                  (a.dst.s0 % 2 == 0);
+  a.tiles_x = (int)((a.E2 + C::BN - 1) / C::BN);
+  a.tiles_y = (int)((a.E1 + C::BM - 1) / C::BM);
+  a.ntiles = (int64_t)a.tiles_x * a.tiles_y * set_ranges(a, (a.E0 + C::ZCH - 1) / C::ZCH, C::ZCH, a.E0, C::H);
+  if (a.ntiles == 0) return cudaSuccess;
+  CUtensorMap tmap;
+  if (!make_tmap(a, C::TP, C::RIN, &tmap)) return cudaErrorNotSupported;
+  cudaError_t e = cudaFuncSetAttribute(k_tile3d_tb, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
+  if (e != cudaSuccess) return e;
+  int occ = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_tile3d_tb, C::NT, C::SMEM);
+  if (e != cudaSuccess) return e;
+  int64_t grid = cap_grid(a, (int64_t)(occ < 1 ? 1 : occ) * num_sms());
+  if (grid > a.ntiles) grid = a.ntiles;
+  return launch_pdl(a.pdl != 0, k_tile3d_tb, grid, C::NT, C::SMEM, st, a, tc_mask, tmap);
+}
+
 using Tile3D3 = Tile3DCfg<3, 8, 2, 2, 5, 32>;      // CTA 64 x 32 outputs, 4 DMMA warps, 5-plane ring, 32 planes per item
 using Tile3D3b = Tile3DCfg<3, 4, 4, 1, 5, 32, 2>;  // CTA 64 x 32, 4 warps of 4 block rows x 2 column groups
 using Tile3D3c = Tile3DCfg<3, 8, 2, 4, 6, 32>;     // CTA 64 x 64 outputs, 8 DMMA warps, 6-plane ring
@@ -929,7 +1161,7 @@ static cudaError_t launch_tile1d(int nk, const S2RArgs& a, cudaStream_t st) {
 
 bool tile_kernel_exists(int ndim, int nk) {
   return (ndim == 1 && (nk & 1) && nk >= 3 && nk <= 31) ||
-         (ndim == 2 && (nk & 1) && nk >= 3 && nk <= 13) || (ndim == 3 && nk == 3);
+         (ndim == 2 && (nk & 1) && nk >= 3 && nk <= 13) || (ndim == 3 && (nk == 3 || nk == 5));
 }
 
 template <class C>
@@ -977,6 +1209,7 @@ static cudaError_t launch_tile3d_cfg(S2RArgs a, int tc_mask, cudaStream_t st) {
 cudaError_t launch_tile(int ndim, int nk, const S2RArgs& a, cudaStream_t st) {
   if (ndim == 1) return launch_tile1d(nk, a, st);
   if (ndim == 3) {
+    if (nk == 5) return launch_tile3d_tb<Tile3DTB>(a, a.tc_mask, st);  // Tf = 2, temporal blocking
     if (nk == 3) {
       const char* e = getenv("CSX_TILE3D_VARIANT");
       if (e && e[0] == '1') return launch_tile3d_cfg<Tile3D3b>(a, a.tc_mask, st);

@@ -338,8 +338,10 @@ csx_status build_plan(csx_plan_s* p) {
   // (C3's "multi-step fused" r = 3, Tf = 2 is nk = 13).
   if (p->ndim == 2 && nk > 13)
     return fail(CSX_ERR_UNSUPPORTED, "2D: composed window 2*r*Tf+1 must be <= 13");
-  if (p->ndim == 3 && p->tf != 1)
-    return fail(CSX_ERR_UNSUPPORTED, "3D: only Tf = 1 (reading A4)");
+  if (p->ndim == 3 && p->tf > 2)
+    return fail(CSX_ERR_UNSUPPORTED, "3D: Tf <= 2 (reading A4)");
+  if (p->ndim == 3 && p->tf == 2 && p->radius != 1)
+    return fail(CSX_ERR_UNSUPPORTED, "3D: Tf = 2 (temporal blocking) needs radius 1");
   for (int a = 0; a < 3; ++a)
     if ((a >= 3 - p->ndim) && p->E[a] < nk)
       return fail(CSX_ERR_INVALID_ARGUMENT, "extent smaller than the composed window 2*r*Tf+1");

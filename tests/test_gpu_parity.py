@@ -254,6 +254,38 @@ def test_full_size_sampled(csx, name, ext, T, tf):
     assert np.max(np.abs(vals - ref)) / np.max(np.abs(got)) <= TOL, info
 
 
+@pytest.mark.parametrize("name", ["heat3d", "box3d27p"])
+@pytest.mark.parametrize("bc", ["fixed", "periodic"])
+def test_parity_3d_two_step_blocking(csx, name, bc):
+    """3D Tf = 2 (k_tile3d_tb: the base stencil run twice per pass through a step-1 plane ring in
+    shared memory): ragged tiles and z chunks, T even / odd (remainder pass of Tf = 1), thin grids,
+    both boundaries, the dense first-pass source."""
+    s = synth.SHAPES[name]
+    w = synth.random_weights(name)
+    for ext in ((40, 50, 70), (70, 37, 45), (9, 130, 66), (33, 5, 200)):
+        u0 = synth.grid(ext, seed=81)
+        for T in (2, 5, 8):
+            got, info = run_gpu(csx, u0, w, s.kind, bc, T, engine="tc_tile", fuse_steps=2)
+            assert info["fuse_steps"] == 2 and info["engine_name"] == "tc_tile"
+            assert rel(got, oracle.run(u0, w, bc, T)) <= TOL, (name, ext, T, bc)
+    # the overlapped sharded schedule (interior / edge z chunks, halo 2) on one rank
+    import os
+    os.environ["CSX_FORCE_OVERLAP"] = "1"
+    try:
+        u0 = synth.grid((100, 30, 40), seed=82)
+        p = csx.Plan(u0.shape, w, shape=s.kind, bc=bc, fuse_steps=2)
+        comm = csx.csx_comm_create(csx.csx_nccl_unique_id(), 0, 1)
+        d_in = torch.from_numpy(u0).cuda()
+        d_out = torch.empty_like(d_in)
+        p.run_sharded(comm, d_in, d_out, 5, u0.size)
+        torch.cuda.synchronize()
+        csx.csx_comm_destroy(comm)
+        p.close()
+        assert rel(d_out.cpu().numpy(), oracle.run(u0, w, bc, 5)) <= TOL, (name, bc, "sharded")
+    finally:
+        del os.environ["CSX_FORCE_OVERLAP"]
+
+
 @pytest.mark.parametrize("variant", ["0", "1", "2", "3", "8", "9"])
 def test_parity_3d_tile_variants(csx, monkeypatch, variant):
     """Every TC_TILE 3D CTA geometry / DMMA order (CSX_TILE3D_VARIANT), star and box, ragged
