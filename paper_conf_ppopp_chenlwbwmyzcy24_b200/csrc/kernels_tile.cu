@@ -735,10 +735,11 @@ struct Tile3DTB {
   static constexpr int SIN_A = (SIN + 15) / 16 * 16;
   static constexpr int SL1 = BM1 * TP;          // doubles per step-1 plane
   static constexpr int SL1_A = (SL1 + 15) / 16 * 16;
-  static constexpr int STAGES = 5;              // input ring
+  static constexpr int STAGES = 4;              // input ring
+  static constexpr int L1S = 4;                 // step-1 plane ring
   static constexpr int ZCH = 32;
   static constexpr int H = 2;                   // halo of the pass (R * Tf)
-  static constexpr int SMEM = (STAGES * SIN_A + 3 * SL1_A) * 8 + 128;
+  static constexpr int SMEM = (STAGES * SIN_A + L1S * SL1_A) * 8 + 128;
   static_assert(TP >= 8 * B * U1C + 4 && TP <= 256 && RIN <= 256, "plane geometry");
 };
 
@@ -781,7 +782,7 @@ __global__ void __launch_bounds__(Tile3DTB::NT, 1)
   using C = Tile3DTB;
   extern __shared__ __align__(128) double smem_raw[];
   double* smem = ring_base(smem_raw);
-  double* l1 = smem + C::STAGES * C::SIN_A;  // 3 step-1 planes
+  double* l1 = smem + C::STAGES * C::SIN_A;  // L1S step-1 planes
   __shared__ __align__(8) uint64_t full[C::STAGES], empty[C::STAGES];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   if (tid == 0) {
@@ -853,39 +854,43 @@ __global__ void __launch_bounds__(Tile3DTB::NT, 1)
     };
     wait_in(z0 - 2);
     wait_in(z0 - 1);
-    for (int64_t zl = z0 - 1; zl <= z1; ++zl) {
-      wait_in(zl + 1);
-      // ---- level 1: step-1 plane zl on the grown tile (rows y0-1 .., cols x0-2 ..) ----
-      const double* pin[3] = {in_plane(zl - 1), in_plane(zl), in_plane(zl + 1)};
-      double* dl1 = l1 + (int)((zl - (z0 - 1)) % 3) * C::SL1_A;
-      const int64_t gz1 = zl + a.gorg0;
-      const bool zf1 = fixed && (gz1 < 1 || gz1 >= a.GE0 - 1);
-      for (int u = warp; u < C::U1R * C::U1C; u += C::NCW) {
-        const int ur = u / C::U1C, uc = u - (u / C::U1C) * C::U1C;
-        const int r0 = ur * C::A * C::G1, c0 = uc * 8 * C::B;
-        double acc[C::G1][2];
-        tb_window<C::G1>(acc, pin, r0, c0, tc_mask, wf, wz, lane);
+    auto l1_plane = [&](int64_t zl) { return l1 + (int)((zl - (z0 - 1)) % C::L1S) * C::SL1_A; };
+    // Phase k: level 1 writes step-1 plane k (inputs k-1..k+1), level 2 writes output plane k-2
+    // (step-1 planes k-3..k-1, finished in earlier phases); the 4-plane step-1 ring keeps the
+    // two apart, so one barrier per phase orders everything.
+    for (int64_t k = z0 - 1; k <= z1 + 1; ++k) {
+      if (k <= z1) {
+        wait_in(k + 1);
+        // ---- level 1: step-1 plane k on the grown tile (rows y0-1 .., cols x0-2 ..) ----
+        const double* pin[3] = {in_plane(k - 1), in_plane(k), in_plane(k + 1)};
+        double* dl1 = l1_plane(k);
+        const int64_t gz1 = k + a.gorg0;
+        const bool zf1 = fixed && (gz1 < 1 || gz1 >= a.GE0 - 1);
+        for (int u = warp; u < C::U1R * C::U1C; u += C::NCW) {
+          const int ur = u / C::U1C, uc = u - (u / C::U1C) * C::U1C;
+          const int r0 = ur * C::A * C::G1, c0 = uc * 8 * C::B;
+          double acc[C::G1][2];
+          tb_window<C::G1>(acc, pin, r0, c0, tc_mask, wf, wz, lane);
 #pragma unroll
-        for (int j = 0; j < C::G1; ++j) {
-          const int r = r0 + C::A * j + alpha, c = c0 + C::B * g + beta;  // step-1 plane coords
-          double v0 = acc[j][0], v1 = acc[j][1];
-          if (fixed && (zf1 || tile_edge)) {  // held frame points keep the input value
-            const int64_t gy = gy0 - 1 + r, gx = gx0 - 2 + c;
-            const double* ctr = pin[1] + (r + 1) * C::TP + c + 2;
-            const bool yf = zf1 || gy < 1 || gy >= a.GE1 - 1;
-            if (yf || gx < 1 || gx >= a.GE2 - 1) v0 = ctr[0];
-            if (yf || gx + 1 < 1 || gx + 1 >= a.GE2 - 1) v1 = ctr[1];
+          for (int j = 0; j < C::G1; ++j) {
+            const int r = r0 + C::A * j + alpha, c = c0 + C::B * g + beta;  // step-1 plane coords
+            double v0 = acc[j][0], v1 = acc[j][1];
+            if (fixed && (zf1 || tile_edge)) {  // held frame points keep the input value
+              const int64_t gy = gy0 - 1 + r, gx = gx0 - 2 + c;
+              const double* ctr = pin[1] + (r + 1) * C::TP + c + 2;
+              const bool yf = zf1 || gy < 1 || gy >= a.GE1 - 1;
+              if (yf || gx < 1 || gx >= a.GE2 - 1) v0 = ctr[0];
+              if (yf || gx + 1 < 1 || gx + 1 >= a.GE2 - 1) v1 = ctr[1];
+            }
+            *reinterpret_cast<double2*>(dl1 + r * C::TP + c) = make_double2(v0, v1);
           }
-          *reinterpret_cast<double2*>(dl1 + r * C::TP + c) = make_double2(v0, v1);
         }
+        release_in();  // input plane k-1 is not read again
       }
-      release_in();  // input plane zl-1 is not read again
-      asm volatile("bar.sync 1, %0;\n" ::"n"(C::NCW * 32) : "memory");  // step-1 plane zl ready
-      // ---- level 2: output plane zo = zl-1 from step-1 planes zl-2, zl-1, zl ----
-      const int64_t zo = zl - 1;
+      // ---- level 2: output plane zo = k-2 from step-1 planes k-3, k-2, k-1 ----
+      const int64_t zo = k - 2;
       if (zo >= z0) {
-        const double* p1[3] = {l1 + (int)((zl - 2 - (z0 - 1)) % 3) * C::SL1_A,
-                               l1 + (int)((zl - 1 - (z0 - 1)) % 3) * C::SL1_A, dl1};
+        const double* p1[3] = {l1_plane(k - 3), l1_plane(k - 2), l1_plane(k - 1)};
         const int r0 = wm * C::A * C::G2, c0 = wn * 8 * C::B;
         double acc[C::G2][2];
         tb_window<C::G2>(acc, p1, r0, c0, tc_mask, wf, wz, lane);
@@ -914,7 +919,7 @@ __global__ void __launch_bounds__(Tile3DTB::NT, 1)
           }
         }
       }
-      asm volatile("bar.sync 1, %0;\n" ::"n"(C::NCW * 32) : "memory");  // ring slot zl-2 free
+      asm volatile("bar.sync 1, %0;\n" ::"n"(C::NCW * 32) : "memory");  // phase k complete
     }
     release_in();  // input planes z1, z1+1
     release_in();
