@@ -17,6 +17,8 @@ def summarise(path):
         if d.get("Metric Name") != "gpu__time_duration.sum":
             continue
         v = float(d["Metric Value"].replace(",", ""))
+        if v != v:  # ncu reports "nan" for a launch it could not time: skip it
+            continue
         unit = d.get("Metric Unit", "")
         scale = {"nsecond": 1e-3, "ns": 1e-3, "usecond": 1.0, "us": 1.0, "msecond": 1e3, "ms": 1e3,
                  "second": 1e6, "s": 1e6}.get(unit, 1.0)
