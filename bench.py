@@ -559,7 +559,7 @@ def main():
             # host->device and its whole result device->host, but step i+1's H2D and step i-1's
             # D2H (PCIe is full duplex) run on their own streams while step i computes.
             plan.set_graph(False)  # alternating buffers would re-capture every step
-            K = max(args.steps, 6)
+            K = max(args.steps, 12)
             s_in, s_out = torch.cuda.Stream(), torch.cuda.Stream()
             hin = [torch.from_numpy(u0).pin_memory() for _ in range(2)]
             hout = [torch.empty(u0.shape, dtype=torch.float64).pin_memory() for _ in range(2)]
