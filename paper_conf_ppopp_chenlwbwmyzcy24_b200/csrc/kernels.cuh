@@ -42,6 +42,7 @@ struct S2RArgs {
   int pdl = 1;                    // TC_TILE: launch with programmatic dependent launch
   int hold_frame = 0;             // write held (frame) values from the staged tile (Tf = 1)
   int use_tma = 0;                // TC_TILE 2D/3D: stage tiles with one TMA tensor copy
+  int l2hint = 0;                 // TMA loads' L2 eviction priority: 0 normal, 1 last, 2 first
   int64_t tma_x0 = 0, tma_y0 = 0, tma_z0 = 0;  // interior origin in tensor-map coordinates
   int r = 0;
   const double* wbase = nullptr;  // base weights (2r+1)^2
