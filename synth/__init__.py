@@ -61,6 +61,43 @@ def grid(extents, seed: int = SEED, rows: tuple[int, int] | None = None) -> np.n
     return vals.reshape((hi - lo,) + extents[1:])
 
 
+def grid_window(extents, lo, hi, seed: int = SEED) -> np.ndarray:
+    """The box [lo, hi) (one bound per axis, clipped to the grid by the caller) of the same
+    global grid as ``grid(extents)``, without building the whole grid."""
+    extents = tuple(int(e) for e in extents)
+    lo = tuple(int(v) for v in lo)
+    hi = tuple(int(v) for v in hi)
+    shape = tuple(h - l for l, h in zip(lo, hi))
+    out = np.empty(shape, dtype=np.float64)
+    strides = [int(np.prod(extents[a + 1:], dtype=np.int64)) for a in range(len(extents))]
+    for idx in np.ndindex(*shape[:-1]):
+        base = sum((lo[a] + idx[a]) * strides[a] for a in range(len(idx)))
+        out[idx] = uniform01(seed, base + lo[-1], shape[-1])
+    return out
+
+
+def grid_torch(extents, device, seed: int = SEED, chunk: int = 1 << 26):
+    """``grid(extents)`` generated on a torch device (same values, bit for bit): for grids too
+    large to build on the host (the maximum-size parity test).  int64 arithmetic wraps like the
+    uint64 reference; right shifts are made logical with a mask."""
+    import torch
+    extents = tuple(int(e) for e in extents)
+    n = int(np.prod(extents, dtype=np.int64))
+    s64 = lambda v: v - (1 << 64) if v >= 1 << 63 else v  # noqa: E731
+    g, c1, c2 = s64(0x9E3779B97F4A7C15), s64(0xBF58476D1CE4E5B9), s64(0x94D049BB133111EB)
+    shr = lambda z, k: (z >> k) & ((1 << (64 - k)) - 1)  # noqa: E731
+    out = torch.empty(n, dtype=torch.float64, device=device)
+    for lo in range(0, n, chunk):
+        m = min(chunk, n - lo)
+        z = torch.arange(lo, lo + m, dtype=torch.int64, device=device) ^ seed
+        z = z + g
+        z = (z ^ shr(z, 30)) * c1
+        z = (z ^ shr(z, 27)) * c2
+        z = z ^ shr(z, 31)
+        out[lo:lo + m] = shr(z, 11).to(torch.float64) * (2.0 ** -53)
+    return out.view(extents)
+
+
 @dataclass(frozen=True)
 class Shape:
     """One benchmark stencil: name, dimension, radius, star/box footprint."""

@@ -446,3 +446,37 @@ def test_graph_replay(csx, name, ext, T):
     assert torch.equal(outs[1], outs[1])
     assert rel(outs[0].cpu().numpy(), ref) <= TOL
     assert rel(outs[1].cpu().numpy(), oracle.run(u0, w, "fixed", T - 1)) <= TOL
+
+
+def test_max_size_beyond_int32(csx):
+    """Maximum-size case: a 50000 x 50000 Box-2D9P grid (2.5e9 points, 20 GB per buffer, flat
+    indices past 2^31) generated on the device by the same seeded generator, T = 4 (two folded
+    passes of Tf = 2, dense first-pass source, k_band), FIXED.  Sampled outputs (corners, faces,
+    band, interior, indices beyond 2^31) against the oracle run on each point's dependence
+    window (half-width T*r + 1, so the window's own held edge cannot reach the point)."""
+    ext, T, r = (50000, 50000), 4, 1
+    free = torch.cuda.mem_get_info()[0]
+    if free < 100 << 30:
+        pytest.skip(f"needs ~100 GB of free device memory, {free >> 30} GB free")
+    w = synth.random_weights("box2d9p")
+    d_in = synth.grid_torch(ext, "cuda")
+    d_out = torch.empty_like(d_in)
+    p = csx.Plan(ext, w, shape="box", bc="fixed")
+    p.run(d_in, d_out, T)
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(5)
+    pts = [(0, 0), (0, 49999), (49999, 0), (49999, 49999), (1, 1), (2, 3), (49998, 49997),
+           (25000, 1), (1, 30000), (49998, 12345), (45000, 45000), (42950, 33333)]
+    pts += [(int(rng.integers(0, 50000)), int(rng.integers(0, 50000))) for _ in range(12)]
+    h = T * r + 1
+    for y, x in pts:
+        lo = (max(0, y - h), max(0, x - h))
+        hi = (min(ext[0], y + h + 1), min(ext[1], x + h + 1))
+        u0w = synth.grid_window(ext, lo, hi)
+        assert float(d_in[y, x]) == u0w[y - lo[0], x - lo[1]]  # device generator == host generator
+        ref = oracle.run(u0w, w, "fixed", T)[y - lo[0], x - lo[1]]
+        got = float(d_out[y, x])
+        assert abs(got - ref) <= TOL, (y, x, got, ref)  # values in [0, 1): max|u| ~ 1
+    p.close()
+    del d_in, d_out
+    torch.cuda.empty_cache()

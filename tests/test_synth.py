@@ -32,3 +32,17 @@ def test_points_match_paper_names():
     pts = {n: s.points for n, s in synth.SHAPES.items()}
     assert pts == {"heat1d": 3, "1d5p": 5, "heat2d": 5, "box2d9p": 9, "star2d13p": 13,
                    "box2d49p": 49, "heat3d": 7, "box3d27p": 27, "star2d9p": 9, "box2d25p": 25}
+
+
+def test_grid_window_and_torch_generator_match_grid():
+    """The windowed and the torch (device-side) generators reproduce grid() bit for bit."""
+    import torch
+    ext = (37, 41, 29)
+    full = synth.grid(ext)
+    w = synth.grid_window(ext, (3, 5, 7), (20, 41, 28))
+    assert np.array_equal(w, full[3:20, 5:41, 7:28])
+    t = synth.grid_torch(ext, "cpu", chunk=1000).numpy()
+    assert np.array_equal(t, full)
+    big = (3000, 70001)  # flat indices past 2^27, several chunks
+    tb = synth.grid_torch(big, "cpu", chunk=1 << 24)
+    assert np.array_equal(tb[2999, -50:].numpy(), synth.grid_window(big, (2999, 69951), (3000, 70001))[0])
