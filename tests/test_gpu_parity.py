@@ -448,35 +448,44 @@ def test_graph_replay(csx, name, ext, T):
     assert rel(outs[1].cpu().numpy(), oracle.run(u0, w, "fixed", T - 1)) <= TOL
 
 
-def test_max_size_beyond_int32(csx):
-    """Maximum-size case: a 50000 x 50000 Box-2D9P grid (2.5e9 points, 20 GB per buffer, flat
-    indices past 2^31) generated on the device by the same seeded generator, T = 4 (two folded
-    passes of Tf = 2, dense first-pass source, k_band), FIXED.  Sampled outputs (corners, faces,
-    band, interior, indices beyond 2^31) against the oracle run on each point's dependence
-    window (half-width T*r + 1, so the window's own held edge cannot reach the point)."""
-    ext, T, r = (50000, 50000), 4, 1
+@pytest.mark.parametrize("name,ext,T", [("box2d9p", (50000, 50000), 4), ("heat3d", (1400, 1400, 1400), 3),
+                                        ("box3d27p", (1360, 1400, 1410), 2)])
+def test_max_size_beyond_int32(csx, name, ext, T):
+    """Maximum-size cases: 2.5-2.7e9-point grids (20-22 GB per buffer, flat indices past 2^31)
+    generated on the device by the same seeded generator: 2D Box-2D9P (two folded passes of
+    Tf = 2, dense first-pass source, k_band) and 3D Heat-3D / Box-3D27P (z-plane rings), FIXED.
+    Sampled outputs (corners, faces, band, interior, indices beyond 2^31) against the oracle
+    run on each point's dependence window (half-width T*r + 1, so the window's own held edge
+    cannot reach the point)."""
+    s = synth.SHAPES[name]
+    r = s.radius
     free = torch.cuda.mem_get_info()[0]
-    if free < 100 << 30:
-        pytest.skip(f"needs ~100 GB of free device memory, {free >> 30} GB free")
-    w = synth.random_weights("box2d9p")
+    need = 5 * 8 * int(np.prod(ext, dtype=np.int64))
+    if free < need:
+        pytest.skip(f"needs ~{need >> 30} GB of free device memory, {free >> 30} GB free")
+    w = synth.random_weights(name)
     d_in = synth.grid_torch(ext, "cuda")
     d_out = torch.empty_like(d_in)
-    p = csx.Plan(ext, w, shape="box", bc="fixed")
+    p = csx.Plan(ext, w, shape=s.kind, bc="fixed")
     p.run(d_in, d_out, T)
     torch.cuda.synchronize()
     rng = np.random.default_rng(5)
-    pts = [(0, 0), (0, 49999), (49999, 0), (49999, 49999), (1, 1), (2, 3), (49998, 49997),
-           (25000, 1), (1, 30000), (49998, 12345), (45000, 45000), (42950, 33333)]
-    pts += [(int(rng.integers(0, 50000)), int(rng.integers(0, 50000))) for _ in range(12)]
+    nd = len(ext)
+    pts = [tuple(0 for _ in ext), tuple(e - 1 for e in ext), tuple(1 for _ in ext),
+           tuple(e - 2 for e in ext), tuple(e // 2 for e in ext),
+           tuple([1] + [e // 3 for e in ext[1:]]), tuple([e - 2 for e in ext[:-1]] + [7]),
+           tuple(int(e * 0.9) for e in ext)]
+    pts += [tuple(int(rng.integers(0, e)) for e in ext) for _ in range(10)]
     h = T * r + 1
-    for y, x in pts:
-        lo = (max(0, y - h), max(0, x - h))
-        hi = (min(ext[0], y + h + 1), min(ext[1], x + h + 1))
+    for pt in pts:
+        lo = tuple(max(0, c - h) for c in pt)
+        hi = tuple(min(e, c + h + 1) for c, e in zip(pt, ext))
         u0w = synth.grid_window(ext, lo, hi)
-        assert float(d_in[y, x]) == u0w[y - lo[0], x - lo[1]]  # device generator == host generator
-        ref = oracle.run(u0w, w, "fixed", T)[y - lo[0], x - lo[1]]
-        got = float(d_out[y, x])
-        assert abs(got - ref) <= TOL, (y, x, got, ref)  # values in [0, 1): max|u| ~ 1
+        loc = tuple(c - l for c, l in zip(pt, lo))
+        assert float(d_in[pt]) == u0w[loc]  # device generator == host generator
+        ref = oracle.run(u0w, w, "fixed", T)[loc]
+        got = float(d_out[pt])
+        assert abs(got - ref) <= TOL, (name, pt, got, ref)  # values in [0, 1): max|u| ~ 1
     p.close()
     del d_in, d_out
     torch.cuda.empty_cache()
