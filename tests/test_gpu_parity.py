@@ -449,7 +449,7 @@ def test_graph_replay(csx, name, ext, T):
 
 
 @pytest.mark.parametrize("name,ext,T", [("box2d9p", (50000, 50000), 4), ("heat3d", (1400, 1400, 1400), 3),
-                                        ("box3d27p", (1360, 1400, 1410), 2)])
+                                        ("box3d27p", (1360, 1400, 1410), 2), ("heat1d", (2900000000,), 23)])
 def test_max_size_beyond_int32(csx, name, ext, T):
     """Maximum-size cases: 2.5-2.7e9-point grids (20-22 GB per buffer, flat indices past 2^31)
     generated on the device by the same seeded generator: 2D Box-2D9P (two folded passes of
