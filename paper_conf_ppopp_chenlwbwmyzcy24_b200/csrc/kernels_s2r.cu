@@ -84,14 +84,13 @@ __global__ void __launch_bounds__(S2R2D<NK>::NT, 2) k_s2r2d(S2RArgs a) {
   __shared__ double sW[FMA ? 2 * G::KS * 4 * 8 : 1];  // [A|B][k][c] for the FMA variant
   __shared__ __align__(8) uint64_t full[G::RAW_STAGES], empty[G::RAW_STAGES];
   double* raw = smem;                                           // RAW_STAGES x RAW
-  double* sA = raw + G::RAW_STAGES * G::RAW;
-  double* sB = sA + (G::STRIPS + 1) * G::PITCH;
-  uint32_t* sL = reinterpret_cast<uint32_t*>(sB + (G::STRIPS + 1) * G::PITCH);
+  double* sAB = raw + G::RAW_STAGES * G::RAW;                   // AB_BUFS x (A | B)
+  uint32_t* sL = reinterpret_cast<uint32_t*>(sAB + G::AB_BUFS * G::AB);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   constexpr int NC = G::NCW * 32;
   // Zero the tiles once so that the K-padding and pad slots are finite (0 * weight 0 = 0);
   // the LUT packs the A and B offsets of each region element (P.1711-1721).
-  for (int i = tid; i < 2 * (G::STRIPS + 1) * G::PITCH; i += G::NT) sA[i] = 0.0;
+  for (int i = tid; i < G::AB_BUFS * G::AB; i += G::NT) sAB[i] = 0.0;
   for (int i = tid; i < G::NE; i += G::NT) sL[i] = (uint32_t)a.lut[i].y;
   if (FMA)  // W[k][c] from the per-lane fragments: lane l of slice s holds W[4s + l%4][l/4]
     for (int i = tid; i < 2 * G::KS * 32; i += G::NT) {
@@ -132,7 +131,10 @@ __global__ void __launch_bounds__(S2R2D<NK>::NT, 2) k_s2r2d(S2RArgs a) {
     const int ty = (int)(tile / a.tiles_x);
     const int tx = (int)(tile - (int64_t)ty * a.tiles_x);
     s2r_mbar_wait(&full[s], (it / G::RAW_STAGES) & 1);
-    asm volatile("bar.sync 1, %0;\n" ::"r"(NC) : "memory");  // previous tile's A/B reads done
+    // A/B buffer of this tile: last read by tile it-2's tessellation, which every warp finished
+    // before it passed tile it-1's "A/B complete" barrier — no barrier needed here
+    double* sA = sAB + (it % G::AB_BUFS) * G::AB;
+    double* sB = sA + (G::STRIPS + 1) * G::PITCH;
     // implicit stencil2row: scatter the staged region through the LUT (branch-free)
     const double* rs = raw + s * G::RAW + G::ODD;
     for (int x = warp; x < G::RR; x += G::NCW) {

@@ -32,10 +32,15 @@ struct S2R2D {
   static constexpr int ODD = R & 1;
   static constexpr int TPR = (ODD + RC + 1) / 2 * 2;  // raw staged row length (even)
   static constexpr int RAW = RR * TPR;                 // doubles per raw stage
-  static constexpr int RAW_STAGES = 2;
+  // A/B are double-buffered (tile k+1 is scattered while slower warps still run tile k's
+  // tessellation: one CTA barrier per tile).  nk = 7 keeps one raw stage (refilled during the
+  // tessellation) so that two CTAs fit an SM; smaller windows keep two (measured).
+  static constexpr int RAW_STAGES = NK >= 7 ? 1 : 2;
+  static constexpr int AB_BUFS = 2;
+  static constexpr int AB = 2 * (STRIPS + 1) * PITCH;  // doubles per A/B buffer
   static constexpr int NCW = 8;                        // consumer warps
   static constexpr int NT = 32 * (NCW + 1);
-  static constexpr int SMEM = 2 * (STRIPS + 1) * PITCH * 8 + NE * 4 + RAW_STAGES * RAW * 8;
+  static constexpr int SMEM = AB_BUFS * AB * 8 + NE * 4 + RAW_STAGES * RAW * 8;
 };
 
 template <int NK>
