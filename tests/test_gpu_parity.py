@@ -489,3 +489,27 @@ def test_max_size_beyond_int32(csx, name, ext, T):
     p.close()
     del d_in, d_out
     torch.cuda.empty_cache()
+
+
+def test_graph_invalidated_by_engine_change(csx):
+    """A captured graph must not outlive an engine switch: after set_engine the same
+    (d_in, d_out, T) runs the new engine (bitwise equal to a fresh plan of that engine)."""
+    w = synth.random_weights("box2d9p")
+    u0 = synth.grid((200, 260), seed=91)
+    d_in = torch.from_numpy(u0).cuda()
+    out = torch.empty_like(d_in)
+    p = csx.Plan(u0.shape, w, shape="box", bc="fixed")
+    p.set_graph(True)
+    for _ in range(2):
+        p.run(d_in, out, 9)        # eager + capture, then replay (TC_TILE)
+    p.set_engine("direct")
+    p.run(d_in, out, 9)
+    torch.cuda.synchronize()
+    q = csx.Plan(u0.shape, w, shape="box", bc="fixed", engine="direct")
+    ref = torch.empty_like(d_in)
+    q.run(d_in, ref, 9)
+    torch.cuda.synchronize()
+    p.close()
+    q.close()
+    assert torch.equal(out, ref)
+    assert rel(out.cpu().numpy(), oracle.run(u0, w, "fixed", 9)) <= TOL
