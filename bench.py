@@ -483,11 +483,13 @@ def main():
         key = f"{args.config}:{engine}"
         if key in tr:
             traffic = tr[key]
+        # the launch-list name of the dominant kernel (k_tile2d / k_s2r3d / k_direct1d ...)
+        kname = f"k_{ {'tc_tile': 'tile', 'tc_s2r': 's2r'}.get(engine, engine)}{s.ndim}d<nk={nk}>"
         if tc_bound:
             achieved = flops / avg_s / 1e12
             roof = {"bound": "tensor", "achieved": achieved, "peak": dmma, "unit": "TFLOP/s",
                     "frac": achieved / dmma, "traffic": traffic, "peak_source": dmma_src,
-                    "kernel": f"k_{engine}{s.ndim}d<{nk}>", "avg_launch_ms": avg_s * 1e3,
+                    "kernel": kname, "avg_launch_ms": avg_s * 1e3,
                     "launches": tc_launches,
                     "per_launch": f"{mma:.0f} DMMA.8x8x4 x 512 flop (Eq 13)",
                     "hbm_frac": byts / avg_s / 1e9 / hbm}
@@ -495,7 +497,7 @@ def main():
             achieved = byts / avg_s / 1e9
             roof = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
                     "frac": achieved / hbm, "traffic": traffic, "peak_source": hbm_src,
-                    "kernel": f"k_{engine}{s.ndim}d<{nk}>", "avg_launch_ms": avg_s * 1e3,
+                    "kernel": kname, "avg_launch_ms": avg_s * 1e3,
                     "launches": tc_launches,
                     "per_launch": f"16 B x {local_points} points (1 read + 1 write per pass)",
                     "tensor_frac": flops / avg_s / 1e12 / dmma}
