@@ -5,7 +5,7 @@
 // same chip" for the 1D and 3D configs (DMMA and DFMA share one FP64 datapath on B200,
 // DESIGN.md §7).
 //
-//   * k_direct1d<R>: every warp owns a window of 32*V consecutive points (V per lane, loaded
+//   * k_direct1d<R, V, PF>: every warp owns a window of 32*V consecutive points (V per lane, loaded
 //     with LDG.128) and runs the Tf fused steps in registers; the R neighbours across lanes come
 //     from warp shuffles.  The error front of the window edges moves R points per step, so the
 //     inner 32 V - 2 hp points (hp = R Tf rounded up to even) are exact and stored.
@@ -19,6 +19,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <cstdlib>
 #include <type_traits>
 
 #include "csx_run.h"
@@ -30,7 +31,7 @@ struct Direct1DW {
   double w[7];
 };
 
-template <int R, int V>
+template <int R, int V, bool PF>
 __global__ void __launch_bounds__(128) k_direct1d(DirectArgs a, Direct1DW W) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -41,16 +42,37 @@ __global__ void __launch_bounds__(128) k_direct1d(DirectArgs a, Direct1DW W) {
   const int64_t N = a.E[2];
   const int64_t nseg = (N + OUT - 1) / OUT;
   const int64_t G = a.GE[2];
+  // PF: the next segment's window is loaded into registers before this one is computed, so
+  // a warp's HBM latency overlaps its own Tf steps of DFMA
+  double2 nxt[PF ? V / 2 : 1];
+  if (PF && gw < nseg) {
+    const double2* src = reinterpret_cast<const double2*>(a.src.p + gw * OUT - hp + lane * V);
+#pragma unroll
+    for (int i = 0; i < V / 2; ++i) nxt[i] = src[i];
+  }
   for (int64_t sg = gw; sg < nseg; sg += nw) {
     const int64_t s0 = sg * OUT;
     const int64_t w0 = s0 - hp + lane * V;  // local index of x[0]
-    const double2* src = reinterpret_cast<const double2*>(a.src.p + w0);
     double x[V];
+    if (PF) {
 #pragma unroll
-    for (int i = 0; i < V / 2; ++i) {
-      const double2 v = src[i];
-      x[2 * i] = v.x;
-      x[2 * i + 1] = v.y;
+      for (int i = 0; i < V / 2; ++i) {
+        x[2 * i] = nxt[i].x;
+        x[2 * i + 1] = nxt[i].y;
+      }
+      if (sg + nw < nseg) {
+        const double2* src = reinterpret_cast<const double2*>(a.src.p + (sg + nw) * OUT - hp + lane * V);
+#pragma unroll
+        for (int i = 0; i < V / 2; ++i) nxt[i] = src[i];
+      }
+    } else {
+      const double2* src = reinterpret_cast<const double2*>(a.src.p + w0);
+#pragma unroll
+      for (int i = 0; i < V / 2; ++i) {
+        const double2 v = src[i];
+        x[2 * i] = v.x;
+        x[2 * i + 1] = v.y;
+      }
     }
     const int64_t g0 = a.gorg[2] + w0;  // global index of x[0]
     // lanes whose points are all at least R from both global ends skip the per-point hold test
@@ -114,22 +136,43 @@ __global__ void __launch_bounds__(128) k_direct1d(DirectArgs a, Direct1DW W) {
 
 bool direct1d_exists(int r, int tf) { return r >= 1 && r <= 3 && tf >= 1 && r * tf <= 16; }
 
-template <int R>
-static cudaError_t launch_d1(const DirectArgs& a, const double* w_host, cudaStream_t st) {
-  constexpr int V = 16;
+template <int R, int V, bool PF>
+static cudaError_t launch_d1v(const DirectArgs& a, const double* w_host, cudaStream_t st) {
   Direct1DW W;
   for (int i = 0; i < 7; ++i) W.w[i] = i <= 2 * R ? w_host[i] : 0.0;
   const int hp = (R * a.tf + 1) & ~1;
+  if (32 * V - 2 * hp <= 0) return cudaErrorNotSupported;
   const int64_t nseg = (a.E[2] + (32 * V - 2 * hp) - 1) / (32 * V - 2 * hp);
   int occ = 0;
-  cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_direct1d<R, V>, 128, 0);
+  cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_direct1d<R, V, PF>, 128, 0);
   if (e != cudaSuccess) return e;
   int64_t grid = (int64_t)(occ < 1 ? 1 : occ) * num_sms();
   const int64_t need = (nseg + 3) / 4;
   if (grid > need) grid = need;
   if (grid < 1) return cudaSuccess;
-  k_direct1d<R, V><<<(unsigned)grid, 128, 0, st>>>(a, W);
+  k_direct1d<R, V, PF><<<(unsigned)grid, 128, 0, st>>>(a, W);
   return cudaGetLastError();
+}
+
+// V points per lane: CSX_DIRECT1D_V = 4 / 8 / 16 / 32; CSX_DIRECT1D_PF = 0 / 1 (register
+// prefetch of the next segment).  Default V = 8 without prefetch, measured (profiles/r01/
+// direct1d_sweep.txt): Heat-1D Tf = 11 2686 GSt/s (V = 16: 1958, V = 4: 2236, V = 8 + PF: 2463),
+// 1D5P Tf = 5 1323 (V = 16: 925) — 72 registers instead of 126 doubles the resident warps.
+template <int R>
+static cudaError_t launch_d1(const DirectArgs& a, const double* w_host, cudaStream_t st) {
+  static int v = -1, pf = -1;
+  if (v < 0) {
+    const char* e = getenv("CSX_DIRECT1D_V");
+    v = e ? atoi(e) : 8;
+    const char* f = getenv("CSX_DIRECT1D_PF");
+    pf = f ? atoi(f) : 0;
+  }
+  const int hp = (R * a.tf + 1) & ~1;
+  if (v == 4 && 2 * hp < 128) return pf ? launch_d1v<R, 4, true>(a, w_host, st) : launch_d1v<R, 4, false>(a, w_host, st);
+  if (v == 16) return pf ? launch_d1v<R, 16, true>(a, w_host, st) : launch_d1v<R, 16, false>(a, w_host, st);
+  if (v == 32) return pf ? launch_d1v<R, 32, true>(a, w_host, st) : launch_d1v<R, 32, false>(a, w_host, st);
+  if (2 * hp < 256) return pf ? launch_d1v<R, 8, true>(a, w_host, st) : launch_d1v<R, 8, false>(a, w_host, st);
+  return pf ? launch_d1v<R, 16, true>(a, w_host, st) : launch_d1v<R, 16, false>(a, w_host, st);
 }
 
 cudaError_t launch_direct1d(const DirectArgs& a, const double* w_host, cudaStream_t st) {
