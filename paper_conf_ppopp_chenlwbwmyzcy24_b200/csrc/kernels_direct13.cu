@@ -32,7 +32,7 @@ struct Direct1DW {
 };
 
 template <int R, int V, bool PF>
-__global__ void __launch_bounds__(128) k_direct1d(DirectArgs a, Direct1DW W) {
+__global__ void __launch_bounds__(128, (V <= 8 ? 8 : 1)) k_direct1d(DirectArgs a, Direct1DW W) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
