@@ -157,7 +157,8 @@ static cudaError_t launch_d1v(const DirectArgs& a, const double* w_host, cudaStr
 // V points per lane: CSX_DIRECT1D_V = 4 / 8 / 16 / 32; CSX_DIRECT1D_PF = 0 / 1 (register
 // prefetch of the next segment).  Default V = 8 without prefetch, measured (profiles/r01/
 // direct1d_sweep.txt): Heat-1D Tf = 11 2686 GSt/s (V = 16: 1958, V = 4: 2236, V = 8 + PF: 2463),
-// 1D5P Tf = 5 1323 (V = 16: 925) — 72 registers instead of 126 doubles the resident warps.
+// 1D5P Tf = 5 1323 (V = 16: 925) — 72 registers instead of 126 doubles the resident warps;
+// __launch_bounds__ min 8 CTAs (64 registers) adds ~1.5 % (2727 / 1335).
 template <int R>
 static cudaError_t launch_d1(const DirectArgs& a, const double* w_host, cudaStream_t st) {
   static int v = -1, pf = -1;
