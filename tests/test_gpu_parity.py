@@ -513,3 +513,41 @@ def test_graph_invalidated_by_engine_change(csx):
     q.close()
     assert torch.equal(out, ref)
     assert rel(out.cpu().numpy(), oracle.run(u0, w, "fixed", 9)) <= TOL
+
+
+_D1_VARIANT_SCRIPT = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+import oracle, synth
+import paper_conf_ppopp_chenlwbwmyzcy24_b200 as csx
+worst = 0.0
+for r, tf, n, T in [(1, 1, 9001, 13), (1, 11, 20000, 25), (2, 5, 7777, 12), (3, 5, 4099, 11), (1, 15, 3000, 33)]:
+    w = synth.random_signed_weights(1, r, seed=60 + r)
+    u0 = synth.grid((n,), seed=61)
+    for bc in ("fixed", "periodic"):
+        p = csx.Plan(u0.shape, w, shape="box", bc=bc, fuse_steps=tf, engine="direct")
+        d_in = torch.from_numpy(u0).cuda()
+        d_out = torch.empty_like(d_in)
+        p.run(d_in, d_out, T)
+        torch.cuda.synchronize()
+        ref = oracle.run(u0, w, bc, T)
+        worst = max(worst, float(np.max(np.abs(d_out.cpu().numpy() - ref)) / np.max(np.abs(ref))))
+        p.close()
+print(worst)
+"""
+
+
+@pytest.mark.parametrize("v,pf", [(4, 0), (4, 1), (8, 1), (16, 0), (16, 1), (32, 0)])
+def test_direct_comparator_1d_variants(v, pf):
+    """Every k_direct1d variant (points per lane V x register prefetch, CSX_DIRECT1D_V /
+    CSX_DIRECT1D_PF; read once per process, hence a subprocess each) matches the oracle; the
+    default (V = 8, no prefetch) is covered by test_direct_comparator_1d_3d."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, CSX_DIRECT1D_V=str(v), CSX_DIRECT1D_PF=str(pf))
+    out = subprocess.run([sys.executable, "-c", _D1_VARIANT_SCRIPT, root], env=env, cwd=root,
+                         capture_output=True, text=True, timeout=300)
+    assert out.returncode == 0, out.stderr[-2000:]
+    assert float(out.stdout.strip().splitlines()[-1]) <= TOL, (v, pf, out.stdout)
