@@ -157,18 +157,12 @@ __global__ void __launch_bounds__(256, (R == 1 ? 2 : 1)) k_direct2d(DirectArgs a
   }
 }
 
-__device__ __forceinline__ double lds64(uint32_t addr) {
-  double v;
-  asm volatile("ld.shared.f64 %0, [%1];\n" : "=d"(v) : "r"(addr));
-  return v;
-}
-
-// One thread's vertical strip: outputs (y, x) for y in [y0, y1) from the shared-memory column at
-// byte address `col` (input (y, x - R + j) at col + 8 (y * pitch + j)); the (2R+1) x (2R+1)
+// One thread's vertical strip: outputs (y, x) for y in [y0, y1) from the shared-memory column
+// `col` (input (y, x - R + j) at col[y * pitch + j]; plain loads the compiler may schedule); the (2R+1) x (2R+1)
 // window slides down the strip with the row loop unrolled by 2R+1 so the rotation is register
 // renaming, not moves; each output sums its taps into two partial accumulators (ILP).
 template <int R, bool EDGE>
-__device__ __forceinline__ void d2_strip(const double* wr, uint32_t col, int pitch, int y0, int y1,
+__device__ __forceinline__ void d2_strip(const double* wr, const double* col, int pitch, int y0, int y1,
                                          double* outc, int64_t opitch, int64_t gy_org, int64_t G1,
                                          bool colhold) {
   constexpr int N = 2 * R + 1;
@@ -176,13 +170,13 @@ __device__ __forceinline__ void d2_strip(const double* wr, uint32_t col, int pit
 #pragma unroll
   for (int i = 0; i < N - 1; ++i)
 #pragma unroll
-    for (int j = 0; j < N; ++j) win[i][j] = lds64(col + 8u * ((y0 - R + i) * pitch + j));
+    for (int j = 0; j < N; ++j) win[i][j] = col[(y0 - R + i) * pitch + j];
   int y = y0;
   for (; y + N <= y1; y += N) {
 #pragma unroll
     for (int u = 0; u < N; ++u) {
 #pragma unroll
-      for (int j = 0; j < N; ++j) win[(u + N - 1) % N][j] = lds64(col + 8u * ((y + u + R) * pitch + j));
+      for (int j = 0; j < N; ++j) win[(u + N - 1) % N][j] = col[(y + u + R) * pitch + j];
       double v0 = 0.0, v1 = 0.0;
 #pragma unroll
       for (int i = 0; i < N; ++i)
@@ -202,7 +196,7 @@ __device__ __forceinline__ void d2_strip(const double* wr, uint32_t col, int pit
   // tail rows (fewer than N): the window is rotated by moves
   for (; y < y1; ++y) {
 #pragma unroll
-    for (int j = 0; j < N; ++j) win[N - 1][j] = lds64(col + 8u * ((y + R) * pitch + j));
+    for (int j = 0; j < N; ++j) win[N - 1][j] = col[(y + R) * pitch + j];
     double v0 = 0.0, v1 = 0.0;
 #pragma unroll
     for (int i = 0; i < N; ++i)
@@ -287,7 +281,9 @@ __global__ void __launch_bounds__(D2WCfg<R, TF>::NT, 1) k_direct2d_ws(DirectArgs
     }
     return;
   }
-  double* lvl[2] = {sm + C::STAGES * C::RY * C::PX, sm + (C::STAGES + 1) * C::RY * C::PX};
+  // offsets from the shared array itself (not pointers picked at run time), so the loads and
+  // stores below stay LDS / STS instead of generic LD / ST
+  const int lvo[2] = {C::STAGES * C::RY * C::PX, (C::STAGES + 1) * C::RY * C::PX};
   double wr[N * N];
 #pragma unroll
   for (int i = 0; i < N * N; ++i) wr[i] = W.w[i];
@@ -302,7 +298,7 @@ __global__ void __launch_bounds__(D2WCfg<R, TF>::NT, 1) k_direct2d_ws(DirectArgs
         : "memory");
     const int ty = (int)(tile / tiles_x), tx = (int)(tile - (int64_t)ty * tiles_x);
     const int64_t oy = (int64_t)ty * C::BY - C::H, ox = (int64_t)tx * C::BX - C::H - C::SH;
-    const double* in = sm + st * C::RY * C::PX;
+    int in_off = st * C::RY * C::PX;
     // edge tiles (touching a FIXED global face) check the frame per point; others skip it
     const int64_t gy_min = a.gorg[1] + oy, gy_max = gy_min + C::RY - 1;
     const int64_t gx_min = a.gorg[2] + ox + C::SH, gx_max = gx_min + C::RX - 1;
@@ -311,7 +307,7 @@ __global__ void __launch_bounds__(D2WCfg<R, TF>::NT, 1) k_direct2d_ws(DirectArgs
 #pragma unroll 1
     for (int s = 1; s <= TF; ++s) {
       const bool last = s == TF;
-      double* out = last ? nullptr : lvl[(s - 1) & 1];
+      const int out_off = last ? 0 : lvo[(s - 1) & 1];
       // one output column per lane (consecutive lanes -> consecutive addresses: conflict-free
       // LDS), a vertical strip of rows per thread with a (2R+1) x (2R+1) sliding window
       const int lo = R * s, hy = C::RY - R * s, hx = C::RX - R * s;
@@ -325,9 +321,9 @@ __global__ void __launch_bounds__(D2WCfg<R, TF>::NT, 1) k_direct2d_ws(DirectArgs
       if (wsr < nws && x < hx && y0 < y1) {
         const int64_t gx = a.gorg[2] + ox + C::SH + x;
         const bool colhold = gx < R || gx >= a.GE[2] - R;
-        const uint32_t col = d2_smem_u32(in + C::SH + x - R);
+        const double* col = sm + in_off + C::SH + x - R;
         if (!last) {
-          double* oc = out + C::SH + x;
+          double* oc = sm + out_off + C::SH + x;
           if (edge) d2_strip<R, true>(wr, col, C::PX, y0, y1, oc, C::PX, a.gorg[1] + oy, a.GE[1], colhold);
           else d2_strip<R, false>(wr, col, C::PX, y0, y1, oc, C::PX, 0, 0, false);
         } else {
@@ -345,7 +341,7 @@ __global__ void __launch_bounds__(D2WCfg<R, TF>::NT, 1) k_direct2d_ws(DirectArgs
         if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(d2_smem_u32(&empty[st])) : "memory");
       }
       asm volatile("bar.sync 1, %0;\n" ::"r"(C::NCW * 32) : "memory");
-      in = out;
+      in_off = out_off;
     }
   }
 }
