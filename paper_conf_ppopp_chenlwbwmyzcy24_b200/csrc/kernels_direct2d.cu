@@ -386,7 +386,7 @@ static cudaError_t launch_d2(const DirectArgs& a, const double* w_host, cudaStre
 }
 
 bool direct2d_exists(int r, int tf) {
-  return (r == 1 && tf >= 1 && tf <= 4) || (r == 2 && tf <= 2) || (r == 3 && tf <= 1);
+  return (r == 1 && tf >= 1 && tf <= 4) || (r == 2 && tf <= 2) || (r == 3 && tf <= 2);
 }
 
 // The base weights travel by value as kernel parameters (constant-bank DFMA operands).
@@ -410,6 +410,8 @@ cudaError_t launch_direct2d(const DirectArgs& a, const double* w_host, cudaStrea
     }
   } else if (a.r == 3 && a.tf == 1) {
     return ws ? launch_d2w<3, 1>(a, w_host, st) : launch_d2<3, 1>(a, w_host, st);
+  } else if (a.r == 3 && a.tf == 2) {  // C3 "multi-step fused" (nk = 13); warp-specialised only
+    return launch_d2w<3, 2>(a, w_host, st);
   }
   return cudaErrorNotSupported;
 }

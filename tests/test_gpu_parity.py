@@ -315,7 +315,7 @@ def test_parity_3d_zchunks(csx, name, engine):
 
 def test_direct_comparator_2d_all_radii(csx):
     """The 2D CUDA-core comparator (k_direct2d) for r = 1..3 and its temporal-blocking depths."""
-    for ndim, r, tf in [(2, 1, 1), (2, 1, 2), (2, 1, 3), (2, 2, 1), (2, 3, 1)]:
+    for ndim, r, tf in [(2, 1, 1), (2, 1, 2), (2, 1, 3), (2, 2, 1), (2, 3, 1), (2, 3, 2)]:
         w = synth.random_signed_weights(ndim, r, seed=40 + r)
         u0 = synth.grid((131, 150), seed=41)
         for bc in ("fixed", "periodic"):
