@@ -49,6 +49,14 @@ CONFIGS = {
     # C3 "multi-step fused" as BASELINE.json words it: r = 3, Tf = 2 (nk = 13, reading A4/A7)
     "star2d13p_10240_tf2": ("star2d13p", (10240, 10240), 100, "fixed", 2),
     "box2d49p_10240_tf2": ("box2d49p", (10240, 10240), 100, "fixed", 2),
+    # 1D well beyond the 126 MB L2 (819 MB per buffer), where HBM binds
+    "heat1d_102400000": ("heat1d", (102400000,), 1000, "fixed", 0),
+    "1d5p_102400000": ("1d5p", (102400000,), 1000, "fixed", 0),
+    # general radius in 3D
+    "box3d125p_512": ("box3d125p", (512, 512, 512), 50, "fixed", 0),
+    "star3d13p_512": ("star3d13p", (512, 512, 512), 50, "fixed", 0),
+    "box3d343p_512": ("box3d343p", (512, 512, 512), 10, "fixed", 0),
+    "star3d19p_512": ("star3d19p", (512, 512, 512), 50, "fixed", 0),
 }
 DEFAULT = "box2d9p_10240"
 METRIC = "FP64 GStencils/s"
@@ -181,7 +189,7 @@ def quiet_stdout():
         os.dup2(2, 1)
 
 
-def algorithmic_mma(ndim, nk, engine, points, tc_planes):
+def algorithmic_mma(ndim, nk, tf, engine, points, tc_planes):
     """DMMA.8x8x4 per pass over `points` outputs: Eq 13 generalised by
     reading A7 (N fragments) and 3D planes for TC_S2R; 4x2/2x4 blocks for TC_TILE 2D/3D and
     8-output Toeplitz blocks (K = nk + 7 rounded up to 4) for TC_TILE 1D."""
@@ -192,7 +200,7 @@ def algorithmic_mma(ndim, nk, engine, points, tc_planes):
         nf = (sw + 7) // 8
         k = nk if ndim == 1 else nk * nk
         return points / (8 * sw) * 2 * math.ceil(k / 4) * nf * tc_planes
-    if engine == "tc_tile" and ndim == 3 and nk == 5:
+    if engine == "tc_tile" and ndim == 3 and tf == 2:
         # 3D Tf = 2 by temporal blocking (k_tile3d_tb): two steps of the base stencil (nk = 3,
         # 4x2 blocks, 6 DMMAs per 64 outputs per TC plane); the recomputed halo is overhead
         return 2 * points / 64 * 6 * tc_planes
@@ -254,7 +262,11 @@ def run_reference(args, cfg_name):
               f"(plain-C oracle, OpenMP {cores} threads)")
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": 1e3 * statistics.median(secs_all) * T / steps, "higher_is_better": True,
+            "ms_per_step": 1e3 * statistics.median(secs_all) * T / steps,
+            "ms_per_step_note": (f"extrapolated to the full T={T} from the {steps} base steps each timed "
+                                 "step runs (the rate is measured; the full-T time is not)"
+                                 if steps < T else "measured"),
+            "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic (splitmix64 seed 20240302, dyadic physical weights)",
             "config": {"workload": cfg_name, "grid": list(ext), "T": T, "bc": bc,
@@ -281,8 +293,10 @@ def main():
     ap.add_argument("--s2r-variant", default="V", choices=["I", "II", "III", "IV", "V"],
                     help="TC_S2R breakdown variant (Fig 6): II CUDA-core tessellation, III no padding/"
                          "no dirty bits, IV padding, V full")
-    ap.add_argument("--exchange", default="peer", choices=["peer", "nccl"],
-                    help="N > 1 halo exchange: SM peer stores over NVLink (default) or NCCL send/recv")
+    ap.add_argument("--exchange", default="both", choices=["both", "peer", "nccl"],
+                    help="N > 1 halo exchange: NCCL send/recv (the north_star path), SM peer stores "
+                         "over NVLink, or both (default: the line's value is the NCCL run, the peer-store "
+                         "run is reported beside it under 'exchange_peer')")
     ap.add_argument("--decomp", default="slab", choices=["slab", "pencil"],
                     help="multi-GPU decomposition: slabs along the slowest axis (default) or a "
                          "p0 x p1 pencil / block grid over the two slowest axes (NCCL exchange; "
@@ -367,7 +381,7 @@ def main():
         lo, hi = plan.shard_box(rank, p0, p1)
         u0 = np.ascontiguousarray(synth.grid(gext, rows=(lo[0], hi[0]))[:, lo[1]:hi[1]])
     elif world > 1:
-        exchange = args.exchange
+        exchange = "peer" if args.exchange == "peer" else "nccl"
         if exchange == "peer":
             # halo exchange by SM peer stores over NVLink (CUDA IPC), epoch flags in peer memory;
             # if the IPC mapping is refused, every rank switches to the NCCL exchange
@@ -449,13 +463,19 @@ def main():
         clk.mark("end")
     ms_total = sum(e0.elapsed_time(e1) for e0, e1 in evs)
     tc_ms, tc_launches, launches = csx.csx_profile_read(plan.handle, reset=True)
-    tc_scale = 1.0  # steps the profiled launches cover, relative to the timed region
+    eager_ms = None  # graph mode: duration of the extra eager (profiled) step
     if graph and args.prof_every > 0:
         csx.csx_profile_enable(plan.handle, args.prof_every)
+        ee0 = torch.cuda.Event(enable_timing=True)
+        ee1 = torch.cuda.Event(enable_timing=True)
+        if flush is not None:
+            flush.fill_(1.0)
+        ee0.record(stream)
         step()
+        ee1.record(stream)
         torch.cuda.synchronize()
+        eager_ms = ee0.elapsed_time(ee1)
         tc_ms, tc_launches, _ = csx.csx_profile_read(plan.handle, reset=True)
-        tc_scale = 1.0 / args.steps
         plan.set_graph(False)
     csx.csx_profile_enable(plan.handle, False)
     if world > 1:
@@ -474,7 +494,16 @@ def main():
     roof = None
     if tc_launches > 0 and engine in ("tc_s2r", "tc_tile"):
         avg_s = tc_ms / tc_launches * 1e-3
-        mma = algorithmic_mma(s.ndim, nk, engine, local_points, tcp)
+        if eager_ms:
+            # graph replay carries no per-kernel events: the dominant kernel's share of the extra
+            # eager step, applied to the replayed step's time (an eager step is slower than its
+            # replay when it is launch-bound, e.g. the 1D configs' short passes)
+            share = min(1.0, tc_ms / eager_ms)
+            avg_eager_ms = tc_ms / tc_launches
+            avg_s = share * ms_step / tc_launches * 1e-3
+        mma = algorithmic_mma(s.ndim, nk, tfm, engine, local_points, tcp)
+        mma_src = ("Eq 13 generalised (reading A7, 3D planes)" if engine == "tc_s2r" else
+                   "TC_TILE block count: K of the a x b output block / 4 per 64 outputs")
         flops = 512.0 * mma
         byts = 16.0 * local_points
         tc_bound = (flops / (dmma * 1e12)) >= (byts / (hbm * 1e9))
@@ -491,7 +520,7 @@ def main():
                     "frac": achieved / dmma, "traffic": traffic, "peak_source": dmma_src,
                     "kernel": kname, "avg_launch_ms": avg_s * 1e3,
                     "launches": tc_launches,
-                    "per_launch": f"{mma:.0f} DMMA.8x8x4 x 512 flop (Eq 13)",
+                    "per_launch": f"{mma:.0f} DMMA.8x8x4 x 512 flop ({mma_src})",
                     "hbm_frac": byts / avg_s / 1e9 / hbm}
         else:
             achieved = byts / avg_s / 1e9
@@ -501,7 +530,15 @@ def main():
                     "launches": tc_launches,
                     "per_launch": f"16 B x {local_points} points (1 read + 1 write per pass)",
                     "tensor_frac": flops / avg_s / 1e12 / dmma}
-        roof["tc_share_of_step"] = tc_ms / (ms_total * tc_scale) if ms_total > 0 else None
+        if eager_ms:
+            roof["tc_share_of_step"] = share
+            roof["timing"] = ("dominant-kernel share of one eager profiled step x the replayed "
+                              "step time / launches per step")
+            roof["avg_launch_ms_eager"] = avg_eager_ms
+            roof["eager_step_ms"] = eager_ms
+        else:
+            roof["tc_share_of_step"] = tc_ms / ms_total if ms_total > 0 else None
+            roof["timing"] = "CUDA events around sampled launches inside the timed steps"
         roof["timed_every"] = args.prof_every
 
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -556,7 +593,8 @@ def main():
             torch.cuda.synchronize()
             ems = e0.elapsed_time(e1) / e_steps
             sync_line = {"value": T * points / (ems * 1e-3) / 1e9, "unit": UNIT, "ms_per_step": ems,
-                         "api": "csx_run_host (pinned host buffers, H2D + run + D2H serialised)"}
+                         "api": "csx_run_host through the C-ABI (pinned host buffers; H2D + run + D2H "
+                                "serialised on one stream, timed by CUDA events)"}
             # A stream of grids through the same public calls: every step copies its own input
             # host->device and its whole result device->host, but step i+1's H2D and step i-1's
             # D2H (PCIe is full duplex) run on their own streams while step i computes.
@@ -597,11 +635,13 @@ def main():
             pms = e0.elapsed_time(e1) / K
             if not torch.equal(hout[(K - 1) % 2], ref.cpu()):
                 raise SystemExit("pipelined e2e result differs from the device run")
-            line["e2e"] = {"value": T * points / (pms * 1e-3) / 1e9, "unit": UNIT,
-                           "h2d_bytes_per_step": int(u0.nbytes), "d2h_bytes_per_step": int(u0.nbytes),
-                           "api": "Plan.run (csx_run) + torch pinned copies, pipelined over "
-                                  f"{K} steps: H2D(i+1) and D2H(i-1) overlap run(i)",
-                           "ms_per_step": pms, "serialised": sync_line}
+            sync_line.update({"h2d_bytes_per_step": int(u0.nbytes), "d2h_bytes_per_step": int(u0.nbytes),
+                              "steps": e_steps})
+            sync_line["pipelined"] = {
+                "value": T * points / (pms * 1e-3) / 1e9, "unit": UNIT, "ms_per_step": pms,
+                "api": "Plan.run (csx_run) + torch pinned copies, pipelined over "
+                       f"{K} steps: H2D(i+1) and D2H(i-1) overlap run(i)"}
+            line["e2e"] = sync_line
         else:
             h_in = torch.from_numpy(u0).pin_memory()
             h_out = torch.empty(u0.shape, dtype=torch.float64).pin_memory()
@@ -621,6 +661,41 @@ def main():
                            "h2d_bytes_per_step": int(u0.nbytes), "d2h_bytes_per_step": int(u0.nbytes),
                            "api": "torch pinned copies + csx_run_sharded" + ("_peer" if comm is None else ""),
                            "ms_per_step": ems}
+    if world > 1 and not pencil and args.exchange == "both":
+        # the same weak-scaled step with the halo exchange fused into SM peer stores over NVLink
+        # (csx_run_sharded_peer), timed the same way (max over ranks); the line's value is the
+        # NCCL run above (the north_star path)
+        peer_line = {"exchange": "peer (SM stores into the neighbours' ghost rows over NVLink, epoch flags)"}
+        pplan = csx.Plan(gext, w, shape=s.kind, bc=bc, fuse_steps=tf, engine=args.engine)
+        err = None
+        try:
+            pplan.peer_setup(rank, world)
+        except Exception as e:  # noqa: BLE001  (reported in the JSON line)
+            err = repr(e)
+        errs = [None] * world
+        dist.all_gather_object(errs, err)
+        if any(errs):
+            peer_line["error"] = next(e for e in errs if e)[:200]
+        else:
+            def pstep():
+                pplan.run_sharded_peer(d_in, d_out, T, n_local, stream)
+            for _ in range(args.warmup):
+                pstep()
+            pev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                   for _ in range(args.steps)]
+            barrier_sync()
+            for e0, e1 in pev:
+                e0.record(stream)
+                pstep()
+                e1.record(stream)
+            barrier_sync()
+            t = torch.tensor([sum(a.elapsed_time(b) for a, b in pev)], device=red_dev, dtype=torch.float64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            pms = float(t.item()) / args.steps
+            peer_line.update({"value": T * points / (pms * 1e-3) / 1e9, "unit": UNIT, "ms_per_step": pms})
+        barrier_sync()  # a neighbour's last push writes into this rank's flags: sync before freeing
+        pplan.close()
+        line["exchange_peer"] = peer_line
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_oracle_sample(shape, gext, T, bc, w)
     if rank == 0:

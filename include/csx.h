@@ -95,6 +95,13 @@ csx_status csx_plan_set_engine(csx_plan_t plan, csx_engine engine);
  * INVALID_ARGUMENT (NULL plan); capture / instantiate failures surface as CUDA from csx_run. */
 csx_status csx_plan_set_graph(csx_plan_t plan, int on);
 
+/* Cap the persistent grids of every kernel the plan launches (TC_TILE, TC_S2R, DIRECT) at
+ * max_ctas CTAs (0 = the default: occupancy x SMs).  Results do not depend on it; it exists so
+ * that tests can drive each persistent CTA around its shared-memory ring many times on small
+ * grids (slot reuse, mbarrier phase flips, empty-slot waits), and for tuning.  Invalidates a
+ * captured graph.  Errors: INVALID_ARGUMENT (NULL plan, max_ctas < 0). */
+csx_status csx_plan_set_max_ctas(csx_plan_t plan, int max_ctas);
+
 /* TC_S2R breakdown variants (Fig 6, P.1865-1950), 2D only: padding = 0 uses the bare
  * stencil2row pitch nk*rr (Fig 5's conflicting 266) instead of the conflict-free one (268);
  * dirty_bits = 0 replaces the dirty-bits padding by conditional stores in the LUT copy loop.

@@ -87,13 +87,14 @@ _sig("csx_profile_read", ctypes.c_int, [_vp, ctypes.POINTER(ctypes.c_double), _i
 
 _sig("csx_halo_schedule", ctypes.c_int, [_vp, ctypes.c_int, ctypes.c_int, _i64p, ctypes.POINTER(ctypes.c_int)])
 _sig("csx_plan_set_graph", ctypes.c_int, [_vp, ctypes.c_int])
+_sig("csx_plan_set_max_ctas", ctypes.c_int, [_vp, ctypes.c_int])
 _sig("csx_shard_box", ctypes.c_int, [_vp, ctypes.c_int, ctypes.c_int, ctypes.c_int, _i64p, _i64p])
 _sig("csx_pencil_schedule", ctypes.c_int, [_vp, ctypes.c_int, ctypes.c_int, ctypes.c_int, _i64p,
                                            ctypes.POINTER(ctypes.c_int)])
 _sig("csx_run_sharded_pencil", ctypes.c_int, [_vp, _vp, ctypes.c_int, ctypes.c_int, _vp, _vp,
                                               ctypes.c_int64, _vp])
 
-EXPORTED = ["csx_plan_set_graph", "csx_shard_box", "csx_pencil_schedule", "csx_run_sharded_pencil", "csx_peer_export", "csx_peer_connect", "csx_run_sharded_peer", "csx_auto_fuse_steps", "csx_plan_set_s2r_variant", "csx_halo_schedule", "csx_profile_enable", "csx_profile_read", "csx_plan", "csx_plan_set_engine", "csx_run", "csx_run_host", "csx_comm_create",
+EXPORTED = ["csx_plan_set_graph", "csx_plan_set_max_ctas", "csx_shard_box", "csx_pencil_schedule", "csx_run_sharded_pencil", "csx_peer_export", "csx_peer_connect", "csx_run_sharded_peer", "csx_auto_fuse_steps", "csx_plan_set_s2r_variant", "csx_halo_schedule", "csx_profile_enable", "csx_profile_read", "csx_plan", "csx_plan_set_engine", "csx_run", "csx_run_host", "csx_comm_create",
             "csx_comm_destroy", "csx_nccl_unique_id", "csx_shard_rows", "csx_run_sharded",
             "csx_plan_destroy", "csx_status_string", "csx_last_error", "csx_plan_info",
             "csx_compose_weights", "csx_weight_matrices", "csx_stencil2row_index",
@@ -407,6 +408,11 @@ class Plan:
     def set_graph(self, on: bool = True):
         """CUDA-graph replay of run() for repeated (d_in, d_out, T) (csx_plan_set_graph)."""
         _check(_lib.csx_plan_set_graph(self._h, int(bool(on))), "csx_plan_set_graph")
+
+    def set_max_ctas(self, max_ctas: int):
+        """Cap every persistent grid the plan launches (0 = occupancy x SMs;
+        csx_plan_set_max_ctas).  Results do not depend on it."""
+        _check(_lib.csx_plan_set_max_ctas(self._h, int(max_ctas)), "csx_plan_set_max_ctas")
 
     def shard_box(self, rank: int, p0: int, p1: int):
         return csx_shard_box(self._h, rank, p0, p1)

@@ -202,7 +202,7 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
         a.GE1 = p->E[1];
         a.GE2 = p->E[2];
       }
-      e = launch_tile(p->ndim, ps.nk, a, st);
+      e = launch_tile(p->ndim, p->radius, ps.tf, a, st);
     } else {
       a.frags = ps.d_frags;
       a.s2r_variant = (p->s2r_pad ? 1 : 0) | (p->s2r_dirty ? 2 : 0) | (p->s2r_fma ? 4 : 0);
@@ -225,19 +225,6 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
         const int64_t need = s2r_explicit_elems(ps.nk, c.E[1], c.E[2]);
         if (need > p->s2r_elems) {
           cudaFree(p->d_s2r);
-    cudaFree(p->d_pstage);
-    if (p->g_exec) cudaGraphExecDestroy((cudaGraphExec_t)p->g_exec);
-    if (p->g_stream) cudaStreamDestroy((cudaStream_t)p->g_stream);
-    if (p->peer) {
-      csx_peer_s* q = p->peer;
-      for (void* ptr : q->opened) cudaIpcCloseMemHandle(ptr);
-      cudaFree(q->block);
-      if (q->cs) cudaStreamDestroy((cudaStream_t)q->cs);
-      if (q->ev_edge) cudaEventDestroy((cudaEvent_t)q->ev_edge);
-      if (q->ev_x) cudaEventDestroy((cudaEvent_t)q->ev_x);
-      delete q;
-      p->peer = nullptr;
-    }
           p->d_s2r = nullptr;
           p->s2r_elems = 0;
           CSX_CUDA(cudaMalloc(&p->d_s2r, (size_t)need * sizeof(double)), "cudaMalloc(stencil2row)");
@@ -276,6 +263,7 @@ csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st) 
     d.tile_list = nullptr;
     d.tile_org = nullptr;
     d.band = 0;
+    d.max_ctas = c.max_ctas;
     direct_tile(p->ndim, d.B);
     for (int a2 = 0; a2 < 3; ++a2) d.tiles[a2] = (int)((c.E[a2] + d.B[a2] - 1) / d.B[a2]);
     d.ntiles = (int64_t)d.tiles[0] * d.tiles[1] * d.tiles[2];
@@ -332,7 +320,7 @@ const char* csx_last_error(void) { return g_err.c_str(); }
 static bool engine_ok(const csx_plan_s* p, csx_engine e) {
   for (const auto& ps : p->passes) {
     if (e == CSX_ENGINE_TC_S2R && !ps.s2r_ok) return false;
-    if (e == CSX_ENGINE_TC_TILE && !(ps.tile_ok && tile_kernel_exists(p->ndim, ps.nk))) return false;
+    if (e == CSX_ENGINE_TC_TILE && !(ps.tile_ok && tile_kernel_exists(p->ndim, p->radius, ps.tf))) return false;
   }
   return true;
 }
@@ -507,6 +495,14 @@ csx_status csx_run(csx_plan_t p, const double* d_in, double* d_out, int64_t T, v
   return CSX_OK;
 }
 
+csx_status csx_plan_set_max_ctas(csx_plan_t p, int max_ctas) {
+  if (!p) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL plan");
+  if (max_ctas < 0) return fail(CSX_ERR_INVALID_ARGUMENT, "max_ctas must be >= 0");
+  p->max_ctas = max_ctas;
+  graph_reset(p);
+  return CSX_OK;
+}
+
 csx_status csx_plan_set_graph(csx_plan_t p, int on) {
   if (!p) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL plan");
   p->graph_on = on != 0;
@@ -589,9 +585,29 @@ csx_status csx_plan_destroy(csx_plan_t p) {
     }
     cudaFree(p->d_s2r);
     cudaFree(p->d_pstage);
+    cudaFree(p->d_halo);
+    p->d_s2r = nullptr;
+    p->d_pstage = nullptr;
+    p->d_halo = nullptr;
     if (p->g_exec) cudaGraphExecDestroy((cudaGraphExec_t)p->g_exec);
     if (p->g_stream) cudaStreamDestroy((cudaStream_t)p->g_stream);
-
+    p->g_exec = nullptr;
+    p->g_stream = nullptr;
+    // NVLink peer exchange (comm.cpp): the block holds both slab buffers and the flag words a
+    // neighbour's last k_peer_push writes into, so the caller must have synchronised every rank
+    // (e.g. a barrier after the last csx_run_sharded_peer) before destroying a peer plan.
+    if (p->peer) {
+      csx_peer_s* q = p->peer;
+      if (q->cs) cudaStreamSynchronize((cudaStream_t)q->cs);
+      for (void* ptr : q->opened) cudaIpcCloseMemHandle(ptr);
+      cudaFree(q->block);
+      if (q->cs) cudaStreamDestroy((cudaStream_t)q->cs);
+      if (q->ev_edge) cudaEventDestroy((cudaEvent_t)q->ev_edge);
+      if (q->ev_x) cudaEventDestroy((cudaEvent_t)q->ev_x);
+      delete q;
+      p->peer = nullptr;
+      p->d_sbuf[0] = p->d_sbuf[1] = nullptr;
+    }
     cudaSetDevice(cur);
   }
   delete p;
@@ -687,7 +703,7 @@ csx_status run_local(csx_plan_s* p, const double* d_in, double* d_out, int64_t T
   // the k_band-recomputed band see them), so no pack into the padded layout.  Not in place for a
   // single pass (its tiles would read halos other tiles already overwrote).
   const bool dense_src = p->engine == CSX_ENGINE_TC_TILE && p->ndim >= 2 && p->bc == CSX_BC_FIXED &&
-                         (d_in != d_out || npass > 1) && tile_reads_dense(d_in, p->E[2]);
+                         (d_in != d_out || npass > 1) && tile_reads_dense(d_in, p->E);
   cudaError_t e = cudaSuccess;
   if (!dense_src) {
     e = launch_pack(d_in, b[0], p->E, st);
@@ -710,6 +726,7 @@ csx_status run_local(csx_plan_s* p, const double* d_in, double* d_out, int64_t T
     if (i == 0 && dense_src) c.src = CView{d_in, p->E[1] * p->E[2], p->E[2], 0, 0, 0, p->E[0]};
     c.dst = last ? out : b[cur ^ 1];
     for (int a = 0; a < 3; ++a) { c.E[a] = p->E[a]; c.gorg[a] = 0; }
+    c.max_ctas = p->max_ctas;
     csx_status s = run_pass(p, p->passes[tfp - 1], c, st);
     if (s != CSX_OK) return s;
     if (!last && p->bc == CSX_BC_PERIODIC) {

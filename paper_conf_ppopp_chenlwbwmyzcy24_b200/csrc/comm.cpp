@@ -91,7 +91,10 @@ static csx_status exchange(csx_plan_s* p, csx_comm_s* c, double* base, int a0, i
     slab_rows(p->spad, base, a0, ops[4 * k + 2], (int)ops[4 * k + 3], &ptr, &n);
     if (ops[4 * k] == 0) r = ncclSend(ptr, n, ncclDouble, (int)ops[4 * k + 1], c->comm, st);
     else r = ncclRecv(ptr, n, ncclDouble, (int)ops[4 * k + 1], c->comm, st);
-    if (r != ncclSuccess) return nccl_fail(r, ops[4 * k] == 0 ? "ncclSend" : "ncclRecv");
+    if (r != ncclSuccess) {  // close the group before reporting, so later NCCL calls fail cleanly
+      ncclGroupEnd();
+      return nccl_fail(r, ops[4 * k] == 0 ? "ncclSend" : "ncclRecv");
+    }
   }
   r = ncclGroupEnd();
   if (r != ncclSuccess) return nccl_fail(r, "ncclGroupEnd");
@@ -242,7 +245,8 @@ static csx_status run_sharded_impl(csx_plan_s* p, csx_comm_s* c, csx_peer_s* q, 
   // (CSX_FORCE_OVERLAP=1 exercises the overlapped schedule on a single rank, for tests)
   const char* fo = getenv("CSX_FORCE_OVERLAP");
   const bool overlap = p->engine == CSX_ENGINE_TC_TILE && (nranks > 1 || (fo && fo[0] == '1'));
-  const int max_ctas = overlap ? num_sms() - 2 : 0;  // leave SMs for the exchange kernels
+  int max_ctas = overlap ? num_sms() - 2 : 0;  // leave SMs for the exchange kernels
+  if (p->max_ctas > 0 && (max_ctas == 0 || p->max_ctas < max_ctas)) max_ctas = p->max_ctas;
   cudaStream_t cs = c ? c->cs : (cudaStream_t)q->cs;
   cudaEvent_t ev_edge = c ? c->ev_edge : (cudaEvent_t)q->ev_edge;
   cudaEvent_t ev_x = c ? c->ev_x : (cudaEvent_t)q->ev_x;
@@ -255,6 +259,7 @@ static csx_status run_sharded_impl(csx_plan_s* p, csx_comm_s* c, csx_peer_s* q, 
     pc.dst = last ? out : b[cur ^ 1];
     for (int a = 0; a < 3; ++a) { pc.E[a] = El[a]; pc.gorg[a] = 0; }
     pc.gorg[a0] = lo;
+    pc.max_ctas = p->max_ctas;
     if (!overlap) {
       s = run_pass(p, p->passes[tfp - 1], pc, st);
       if (s != CSX_OK) return s;
@@ -434,7 +439,10 @@ static csx_status exchange_pencil(csx_plan_s* p, csx_comm_s* c, double* base, in
       }
       if (o[1] == 0) r = ncclSend(ptr, n, ncclDouble, (int)o[2], c->comm, st);
       else r = ncclRecv(ptr, n, ncclDouble, (int)o[2], c->comm, st);
-      if (r != ncclSuccess) return nccl_fail(r, o[1] == 0 ? "ncclSend" : "ncclRecv");
+      if (r != ncclSuccess) {
+        ncclGroupEnd();
+        return nccl_fail(r, o[1] == 0 ? "ncclSend" : "ncclRecv");
+      }
     }
     r = ncclGroupEnd();
     if (r != ncclSuccess) return nccl_fail(r, "ncclGroupEnd");
@@ -541,6 +549,7 @@ static csx_status run_sharded_pencil_impl(csx_plan_s* p, csx_comm_s* c, int p0, 
     pc.src = CView{b[cur].p, b[cur].s0, b[cur].s1, pd.O[0], pd.O[1], pd.O[2], pd.A[0]};
     pc.dst = last ? out : b[cur ^ 1];
     for (int a = 0; a < 3; ++a) { pc.E[a] = El[a]; pc.gorg[a] = lo[a]; }
+    pc.max_ctas = p->max_ctas;
     s = run_pass(p, p->passes[tfp - 1], pc, st);
     if (s != CSX_OK) return s;
     if (!last) {

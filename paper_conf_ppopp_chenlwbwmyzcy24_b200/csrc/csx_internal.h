@@ -146,6 +146,7 @@ struct csx_plan_s {
   // CUDA graph replay of csx_run (csx_plan_set_graph): the pass sequence of one
   // (d_in, d_out, T) captured once and replayed with one cudaGraphLaunch
   int graph_on = 0;
+  int max_ctas = 0;                // persistent-grid cap of every launch (csx_plan_set_max_ctas)
   void* g_exec = nullptr;          // cudaGraphExec_t
   void* g_stream = nullptr;        // non-blocking capture stream
   const double* g_in = nullptr;

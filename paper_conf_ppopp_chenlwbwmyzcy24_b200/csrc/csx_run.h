@@ -25,7 +25,7 @@ csx_status ensure_grid(csx_plan_s* p, Padded* pd, double** bufs, const int64_t* 
 csx_status run_pass(csx_plan_s* p, Pass& ps, const PassCtx& c, cudaStream_t st);
 csx_status run_local(csx_plan_s* p, const double* d_in, double* d_out, int64_t T, cudaStream_t st);
 void direct_tile(int ndim, int* B);
-bool tile_kernel_exists(int ndim, int nk);
-bool tile_reads_dense(const double* p, int64_t E2);
+bool tile_kernel_exists(int ndim, int radius, int tf);
+bool tile_reads_dense(const double* p, const int64_t* E);
 
 }  // namespace csx

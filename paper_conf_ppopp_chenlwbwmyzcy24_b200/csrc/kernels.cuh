@@ -66,6 +66,7 @@ struct DirectArgs {
   const int64_t* tile_org;   // band strips: explicit tile origins (3 per tile), or nullptr
   const double* w;      // base weights (2r+1)^ndim dense
   int ndim;
+  int max_ctas = 0;     // cap on the persistent grid (0 = all SMs; csx_plan_set_max_ctas)
 };
 
 // NVLink peer-memory halo push (kernels_peer.cu)
@@ -95,7 +96,8 @@ cudaError_t launch_pack(const double* in, View dst, const int64_t* E, cudaStream
 cudaError_t launch_ghost_fill(View buf, const int64_t* E, const int* real, const int* fill, int H,
                               cudaStream_t st);
 cudaError_t launch_s2r(int ndim, int nk, int nf, const S2RArgs& a, int tc_mask, cudaStream_t st);
-cudaError_t launch_tile(int ndim, int nk, const S2RArgs& a, cudaStream_t st);
+// TC_TILE pass of `tf` fused steps of a base radius `radius` stencil (nk = 2 radius tf + 1)
+cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStream_t st);
 cudaError_t launch_direct(const DirectArgs& a, cudaStream_t st);
 // 2D comparator kernel (kernels_direct2d.cu): compile-time (r, Tf), weights by value.
 bool direct2d_exists(int r, int tf);
@@ -120,5 +122,7 @@ int64_t s2r_explicit_elems(int nk, int64_t E1, int64_t E2);
 cudaError_t launch_s2r_explicit(int nk, CView src, View dst, const int64_t* E, const double* wc,
                                 double* scratch, cudaStream_t st);
 int num_sms();
+// persistent grid size: occupancy x SMs, capped by max_ctas (> 0) and by the work items
+int64_t persistent_grid(int occ, int max_ctas, int64_t items);
 
 }  // namespace csx

@@ -152,8 +152,7 @@ cudaError_t launch_direct(const DirectArgs& a, cudaStream_t st) {
       if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_direct<3>, 256, smem);
   }
   if (e != cudaSuccess) return e;
-  int64_t grid = (int64_t)(occ < 1 ? 1 : occ) * num_sms();
-  if (grid > a.ntiles) grid = a.ntiles;
+  const int64_t grid = persistent_grid(occ, a.max_ctas, a.ntiles);
   switch (a.ndim) {
     case 1: k_direct<1><<<(unsigned)grid, 256, smem, st>>>(a); break;
     case 2: k_direct<2><<<(unsigned)grid, 256, smem, st>>>(a); break;

@@ -146,9 +146,7 @@ static cudaError_t launch_d1v(const DirectArgs& a, const double* w_host, cudaStr
   int occ = 0;
   cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_direct1d<R, V, PF>, 128, 0);
   if (e != cudaSuccess) return e;
-  int64_t grid = (int64_t)(occ < 1 ? 1 : occ) * num_sms();
-  const int64_t need = (nseg + 3) / 4;
-  if (grid > need) grid = need;
+  const int64_t grid = persistent_grid(occ, a.max_ctas, (nseg + 3) / 4);
   if (grid < 1) return cudaSuccess;
   k_direct1d<R, V, PF><<<(unsigned)grid, 128, 0, st>>>(a, W);
   return cudaGetLastError();
@@ -370,8 +368,7 @@ static cudaError_t launch_d3(const DirectArgs& a, const double* w_host, cudaStre
   if (e != cudaSuccess) return e;
   const int64_t nitems = ((a.E[2] + C::BX - 1) / C::BX) * ((a.E[1] + C::BY - 1) / C::BY) *
                          ((a.E[0] + C::ZC - 1) / C::ZC);
-  int64_t grid = (int64_t)(occ < 1 ? 1 : occ) * num_sms();
-  if (grid > nitems) grid = nitems;
+  const int64_t grid = persistent_grid(occ, a.max_ctas, nitems);
   if (grid < 1) return cudaSuccess;
   k_direct3d<R><<<(unsigned)grid, C::NT, C::SMEM, st>>>(a, W);
   return cudaGetLastError();

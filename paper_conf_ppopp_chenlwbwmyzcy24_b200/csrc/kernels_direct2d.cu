@@ -359,8 +359,7 @@ static cudaError_t launch_d2w(const DirectArgs& a, const double* w_host, cudaStr
   int occ = 0;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_direct2d_ws<R, TF>, C::NT, C::SMEM);
   if (e != cudaSuccess) return e;
-  int64_t grid = (int64_t)(occ < 1 ? 1 : occ) * num_sms();
-  if (grid > b.ntiles) grid = b.ntiles;
+  const int64_t grid = persistent_grid(occ, a.max_ctas, b.ntiles);
   k_direct2d_ws<R, TF><<<(unsigned)grid, C::NT, C::SMEM, st>>>(b, W);
   return cudaGetLastError();
 }
@@ -379,23 +378,29 @@ static cudaError_t launch_d2(const DirectArgs& a, const double* w_host, cudaStre
   int occ = 0;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_direct2d<R, TF>, C::NT, C::SMEM);
   if (e != cudaSuccess) return e;
-  int64_t grid = (int64_t)(occ < 1 ? 1 : occ) * num_sms();
-  if (grid > b.ntiles) grid = b.ntiles;
+  const int64_t grid = persistent_grid(occ, a.max_ctas, b.ntiles);
   k_direct2d<R, TF><<<(unsigned)grid, C::NT, C::SMEM, st>>>(b, W);
   return cudaGetLastError();
 }
 
+static int direct_ws() {
+  static const int ws = [] {
+    const char* e = getenv("CSX_DIRECT_WS");
+    return e ? atoi(e) : 1;
+  }();
+  return ws;
+}
+
+// r = 3, Tf = 2 (C3 "multi-step fused", nk = 13) exists only as the warp-specialised kernel:
+// with CSX_DIRECT_WS=0 it reports unsupported, so the generic direct kernel runs instead
 bool direct2d_exists(int r, int tf) {
-  return (r == 1 && tf >= 1 && tf <= 4) || (r == 2 && tf <= 2) || (r == 3 && tf <= 2);
+  return (r == 1 && tf >= 1 && tf <= 4) || (r == 2 && tf <= 2) || (r == 3 && tf == 1) ||
+         (r == 3 && tf == 2 && direct_ws());
 }
 
 // The base weights travel by value as kernel parameters (constant-bank DFMA operands).
 cudaError_t launch_direct2d(const DirectArgs& a, const double* w_host, cudaStream_t st) {
-  static int ws = -1;
-  if (ws < 0) {
-    const char* e = getenv("CSX_DIRECT_WS");
-    ws = e ? atoi(e) : 1;
-  }
+  const int ws = direct_ws();
   if (a.r == 1) {
     switch (a.tf) {
       case 1: return ws ? launch_d2w<1, 1>(a, w_host, st) : launch_d2<1, 1>(a, w_host, st);
@@ -410,7 +415,7 @@ cudaError_t launch_direct2d(const DirectArgs& a, const double* w_host, cudaStrea
     }
   } else if (a.r == 3 && a.tf == 1) {
     return ws ? launch_d2w<3, 1>(a, w_host, st) : launch_d2<3, 1>(a, w_host, st);
-  } else if (a.r == 3 && a.tf == 2) {  // C3 "multi-step fused" (nk = 13); warp-specialised only
+  } else if (a.r == 3 && a.tf == 2 && ws) {  // C3 "multi-step fused" (nk = 13)
     return launch_d2w<3, 2>(a, w_host, st);
   }
   return cudaErrorNotSupported;

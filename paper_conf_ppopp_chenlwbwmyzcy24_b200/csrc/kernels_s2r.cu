@@ -364,6 +364,13 @@ __global__ void __launch_bounds__(128, 3) k_s2r3d(S2RArgs a, int tc_mask) {
 }
 
 // ------------------------------------------------------------------------------------------
+int64_t persistent_grid(int occ, int max_ctas, int64_t items) {
+  int64_t grid = (int64_t)(occ < 1 ? 1 : occ) * num_sms();
+  if (max_ctas > 0 && grid > max_ctas) grid = max_ctas;
+  if (grid > items) grid = items;
+  return grid;
+}
+
 int num_sms() {
   static int n = 0;
   if (n == 0) {
@@ -384,8 +391,7 @@ static cudaError_t launch_persistent(K kernel, int smem, int nthreads, int64_t i
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, nthreads, smem);
   if (e != cudaSuccess) return e;
   if (occ < 1) return cudaErrorInvalidConfiguration;
-  int64_t grid = (int64_t)occ * num_sms();
-  if (grid > items) grid = items;
+  int64_t grid = persistent_grid(occ, a.max_ctas, items);
   if (grid < 1) grid = 1;
   kernel<<<(unsigned)grid, nthreads, smem, st>>>(a);
   return cudaGetLastError();
@@ -456,8 +462,7 @@ cudaError_t launch_s2r(int ndim, int nk, int nf, const S2RArgs& a, int tc_mask, 
     int occ = 0;
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 128, smem);
     if (e != cudaSuccess) return e;
-    int64_t grid = (int64_t)(occ < 1 ? 1 : occ) * num_sms();
-    if (grid > a.ntiles) grid = a.ntiles;
+    const int64_t grid = persistent_grid(occ, a.max_ctas, a.ntiles);
     kern<<<(unsigned)grid, 128, smem, st>>>(a, tc_mask);
     return cudaGetLastError();
   }

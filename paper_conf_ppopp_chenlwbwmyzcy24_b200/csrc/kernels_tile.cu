@@ -173,19 +173,19 @@ static bool make_tmap(S2RArgs& a, int bx, int by, CUtensorMap* map) {
 // Host: can the TC_TILE 2D / 3D kernels stage their tiles straight from a DENSE grid (the user's
 // d_in: no ghost cells, row pitch E2)?  The TMA tensor map zero-fills the halo boxes that fall
 // outside the grid, which only the held FIXED frame and the band recomputed by k_band could see.
-bool tile_reads_dense(const double* p, int64_t E2) {
+// Decided by a trial encode of the dense geometry (the kernels' boxes are <= 256 x 256, which
+// the encoder accepts whenever it accepts the geometry), so a rejected map falls back to the
+// pack instead of failing the pass.
+bool tile_reads_dense(const double* p, const int64_t* E) {
   const char* e = getenv("CSX_TMA");
   if (e && e[0] == '0') return false;
   const char* d = getenv("CSX_DENSE_SRC");
   if (d && d[0] == '0') return false;
-  void* fn = nullptr;
-  cudaDriverEntryPointQueryResult q;
-  if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess ||
-      q != cudaDriverEntryPointSuccess) {
-    cudaGetLastError();
-    return false;
-  }
-  return (reinterpret_cast<uintptr_t>(p) & 15) == 0 && E2 % 2 == 0;
+  if ((reinterpret_cast<uintptr_t>(p) & 15) != 0 || E[2] % 2 != 0) return false;
+  S2RArgs a;
+  a.src = CView{p, E[1] * E[2], E[2], 0, 0, 0, E[0]};
+  CUtensorMap map;
+  return make_tmap(a, 8, 8, &map);
 }
 
 // Programmatic dependent launch (sm_90+): the kernels below are launched with programmatic
@@ -256,10 +256,6 @@ static cudaError_t launch_pdl(bool pdl, void (*k)(KArgs...), int64_t grid, int n
   return cudaLaunchKernelEx(&cfg, k, args...);
 }
 
-static int64_t cap_grid(const S2RArgs& a, int64_t grid) {
-  if (a.max_ctas > 0 && grid > a.max_ctas) grid = a.max_ctas;
-  return grid;
-}
 
 constexpr int s2r_pitch_dev(int min_pitch) {
   int p = min_pitch;
@@ -514,10 +510,17 @@ static int tile_variant() {
 // DMMA warps compute output plane zo from the NK staged planes zo-R .. zo+R (every tensor-core z
 // offset is a K-slice group of the same GEMM; single-tap z offsets — the star arms, reading A9 —
 // are DFMAs on the same staged planes), then release plane zo-R, which no later output needs.
-template <int NK_, int G_, int WM_, int WN_, int STAGES_, int ZCH_, int CG_ = 1, int KO_ = 0>
+//
+// Radius 2 / 3 (nk = 5 / 7, §8(f)#2) use the same kernel with the planner's block shape for the
+// window (2x4 for nk = 5, 4x2 for nk = 7: the smaller K, as in 2D) and, where NK x KS weight
+// fragments would not fit the register file (WREG = 0, nk = 7: 7 x 20), each TC plane's KS
+// fragments loaded from L1 just before its GEMM (KS loads per G*KS DMMAs).
+template <int NK_, int G_, int WM_, int WN_, int STAGES_, int ZCH_, int CG_ = 1, int KO_ = 0,
+          int A_ = 4, int B_ = 2, int WREG_ = 1>
 struct Tile3DCfg {
-  static constexpr int NK = NK_, A = 4, B = 2, KC = 4 * ((2 + NK - 1 + 3) / 4), G = G_, WM = WM_,
+  static constexpr int NK = NK_, A = A_, B = B_, KC = 4 * ((B_ + NK - 1 + 3) / 4), G = G_, WM = WM_,
                        WN = WN_, STAGES = STAGES_, ZCH = ZCH_, CG = CG_;
+  static constexpr int WREG = WREG_;  // 1: all planes' weight fragments live in registers
   // DMMA issue order inside a TC plane: 0 = by input row (an A fragment feeds every block whose
   // window holds the row; consecutive DMMAs often hit the same accumulator chain), 1 = k-slice
   // outer, blocks inner (G independent chains between dependent DMMAs; one LDS per DMMA)
@@ -595,12 +598,13 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
   }
   const int wm = warp / C::WN, wn = warp - (warp / C::WN) * C::WN;
   const int g = lane >> 2, t = lane & 3;
-  double wf[C::NK][C::KS];
+  double wf[C::WREG ? C::NK : 1][C::KS];
   double wz[C::NK];
 #pragma unroll
   for (int p = 0; p < C::NK; ++p) {
+    if (C::WREG)
 #pragma unroll
-    for (int k = 0; k < C::KS; ++k) wf[p][k] = a.frags[(p * C::KS + k) * 32 + lane];
+      for (int k = 0; k < C::KS; ++k) wf[C::WREG ? p : 0][k] = a.frags[(p * C::KS + k) * 32 + lane];
     wz[p] = a.wc[(p * C::NK + C::R) * C::NK + C::R];
   }
   const int alpha = (2 * t) / C::B, beta = (2 * t) % C::B;
@@ -649,6 +653,11 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
 #pragma unroll
       for (int dz = 0; dz < C::NK; ++dz) {
         const double* stg = smem + slot[dz] * C::STAGE_A;
+        if (!C::WREG && (tc_mask & (1 << dz))) {  // this plane's fragments, from L1
+#pragma unroll
+          for (int k = 0; k < C::KS; ++k) wf[0][k] = __ldg(a.frags + (dz * C::KS + k) * 32 + lane);
+        }
+        const int wp = C::WREG ? dz : 0;
         if ((tc_mask & (1 << dz)) && C::KO == 1) {
           const double* base = stg + lane_off;
 #pragma unroll
@@ -661,7 +670,7 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
                 for (int cg = 0; cg < C::CG; ++cg)
                   dmma_t(acc[cg][j][0], acc[cg][j][1],
                          base[(C::A * j + rho) * C::TP + cg * 8 * C::B + 4 * h],
-                         wf[dz][rho * (C::KC / 4) + h]);
+                         wf[wp][rho * (C::KC / 4) + h]);
         } else if (tc_mask & (1 << dz)) {
           const double* base = stg + lane_off;
 #pragma unroll
@@ -679,7 +688,7 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
                 if (rho >= 0 && rho < C::KR)
 #pragma unroll
                   for (int cg = 0; cg < C::CG; ++cg)
-                    dmma_t(acc[cg][j][0], acc[cg][j][1], f[cg][h], wf[dz][rho * (C::KC / 4) + h]);
+                    dmma_t(acc[cg][j][0], acc[cg][j][1], f[cg][h], wf[wp][rho * (C::KC / 4) + h]);
               }
           }
         } else if (any_cuda && wz[dz] != 0.0) {
@@ -981,8 +990,7 @@ static cudaError_t launch_tile3d_tb(S2RArgs a, int tc_mask, cudaStream_t st) {
   int occ = 0;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_tile3d_tb, C::NT, C::SMEM);
   if (e != cudaSuccess) return e;
-  int64_t grid = cap_grid(a, (int64_t)(occ < 1 ? 1 : occ) * num_sms());
-  if (grid > a.ntiles) grid = a.ntiles;
+  const int64_t grid = persistent_grid(occ, a.max_ctas, a.ntiles);
   return launch_pdl(a.pdl != 0, k_tile3d_tb, grid, C::NT, C::SMEM, st, a, tc_mask, tmap);
 }
 
@@ -992,6 +1000,10 @@ using Tile3D3c = Tile3DCfg<3, 8, 2, 4, 6, 32>;     // CTA 64 x 64 outputs, 8 DMM
 using Tile3D3d = Tile3DCfg<3, 2, 8, 1, 5, 32, 2>;  // CTA 64 x 32, 8 warps of 2 block rows x 2 column groups
 using Tile3D3k = Tile3DCfg<3, 8, 2, 2, 5, 32, 1, 1>;  // Tile3D3, k-slice-outer DMMA order
 using Tile3D3ck = Tile3DCfg<3, 8, 2, 4, 6, 32, 1, 1>;  // Tile3D3c, k-slice-outer DMMA order
+// radius 2: 2x4 blocks (K = 6 x 8), 8 DMMA warps, CTA 32 x 64, 6-plane ring, weights per plane
+using Tile3D5 = Tile3DCfg<5, 4, 4, 2, 6, 32, 1, 0, 2, 4, 0>;
+// radius 3: 4x2 blocks (K = 10 x 8), 8 DMMA warps, CTA 32 x 64, 8-plane ring, weights per plane
+using Tile3D7 = Tile3DCfg<7, 4, 2, 4, 8, 32, 1, 0, 4, 2, 0>;
 
 
 // ------------------------------------------------------------------------------------------
@@ -1170,8 +1182,7 @@ static cudaError_t launch_tile1d_cfg(S2RArgs a, cudaStream_t st) {
   int occ = 0;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_tile1d<C>, C::NT, C::SMEM);
   if (e != cudaSuccess) return e;
-  int64_t grid = cap_grid(a, (int64_t)(occ < 1 ? 1 : occ) * num_sms());
-  if (grid > a.ntiles) grid = a.ntiles;
+  const int64_t grid = persistent_grid(occ, a.max_ctas, a.ntiles);
   return launch_pdl(a.pdl != 0, k_tile1d<C>, grid, C::NT, C::SMEM, st, a);
 }
 
@@ -1220,9 +1231,15 @@ static cudaError_t launch_tile1d(int nk, const S2RArgs& a, cudaStream_t st) {
   return cudaErrorNotSupported;
 }
 
-bool tile_kernel_exists(int ndim, int nk) {
-  return (ndim == 1 && (nk & 1) && nk >= 3 && nk <= 31) ||
-         (ndim == 2 && (nk & 1) && nk >= 3 && nk <= 13) || (ndim == 3 && (nk == 3 || nk == 5));
+// (ndim, base radius, fused steps) -> is there a TC_TILE kernel for the pass?  3D: Tf = 1 runs
+// the per-plane GEMM of the composed window (= the base window) for r = 1..3 (nk = 3, 5, 7);
+// Tf = 2 only by the temporal blocking of the base r = 1 stencil (k_tile3d_tb).
+bool tile_kernel_exists(int ndim, int radius, int tf) {
+  const int nk = 2 * radius * tf + 1;
+  if (ndim == 1) return nk >= 3 && nk <= 31;
+  if (ndim == 2) return nk >= 3 && nk <= 13;
+  if (ndim == 3) return (tf == 1 && radius >= 1 && radius <= 3) || (tf == 2 && radius == 1);
+  return false;
 }
 
 template <class C>
@@ -1242,8 +1259,7 @@ static cudaError_t launch_tile_cfg(S2RArgs a, cudaStream_t st) {
   int occ = 0;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_tile2d<C>, C::NT, C::SMEM);
   if (e != cudaSuccess) return e;
-  int64_t grid = cap_grid(a, (int64_t)(occ < 1 ? 1 : occ) * num_sms());
-  if (grid > a.ntiles) grid = a.ntiles;
+  const int64_t grid = persistent_grid(occ, a.max_ctas, a.ntiles);
   return launch_pdl(a.pdl != 0, k_tile2d<C>, grid, C::NT, C::SMEM, st, a, tmap);
 }
 
@@ -1270,15 +1286,18 @@ static cudaError_t launch_tile3d_cfg(S2RArgs a, int tc_mask, cudaStream_t st) {
   int occ = 0;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_tile3d<C>, C::NT, C::SMEM);
   if (e != cudaSuccess) return e;
-  int64_t grid = cap_grid(a, (int64_t)(occ < 1 ? 1 : occ) * num_sms());
-  if (grid > a.ntiles) grid = a.ntiles;
+  const int64_t grid = persistent_grid(occ, a.max_ctas, a.ntiles);
   return launch_pdl(a.pdl != 0, k_tile3d<C>, grid, C::NT, C::SMEM, st, a, tc_mask, tmap);
 }
 
-cudaError_t launch_tile(int ndim, int nk, const S2RArgs& a, cudaStream_t st) {
+cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStream_t st) {
+  if (!tile_kernel_exists(ndim, radius, tf)) return cudaErrorNotSupported;
+  const int nk = 2 * radius * tf + 1;
   if (ndim == 1) return launch_tile1d(nk, a, st);
   if (ndim == 3) {
-    if (nk == 5) return launch_tile3d_tb<Tile3DTB>(a, a.tc_mask, st);  // Tf = 2, temporal blocking
+    if (tf == 2) return launch_tile3d_tb<Tile3DTB>(a, a.tc_mask, st);  // r = 1: temporal blocking
+    if (nk == 5) return launch_tile3d_cfg<Tile3D5>(a, a.tc_mask, st);
+    if (nk == 7) return launch_tile3d_cfg<Tile3D7>(a, a.tc_mask, st);
     if (nk == 3) {
       const char* e = getenv("CSX_TILE3D_VARIANT");
       if (e && e[0] == '1') return launch_tile3d_cfg<Tile3D3b>(a, a.tc_mask, st);

@@ -140,6 +140,12 @@ SHAPES = {
         Shape("box3d27p", 3, 1, "box", 8),
         Shape("star2d9p", 2, 2, "star", 9),
         Shape("box2d25p", 2, 2, "box", 10),
+        # general radius in 3D (r <= 3 in every dimension; the paper's 3D
+        # method is a sum of per-plane 2D ConvStencils for any plane window, P.1788-1800)
+        Shape("star3d13p", 3, 2, "star", 11),
+        Shape("box3d125p", 3, 2, "box", 12),
+        Shape("star3d19p", 3, 3, "star", 13),
+        Shape("box3d343p", 3, 3, "box", 14),
     ]
 }
 
@@ -168,6 +174,10 @@ def physical_weights(name: str) -> np.ndarray:
         centre, arms = 0.5, [1 / 16, 1 / 16]
     elif name == "heat3d":
         centre, arms = 0.625, [0.0625]
+    elif name == "star3d13p":
+        centre, arms = 0.25, [1 / 16, 1 / 16]
+    elif name == "star3d19p":
+        centre, arms = 0.25, [1 / 16, 1 / 32, 1 / 32]
     else:
         raise KeyError(name)
     w[(c,) * s.ndim] = centre

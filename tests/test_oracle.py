@@ -127,7 +127,8 @@ def test_fourier_decay_heat(name, alpha):
     assert np.max(np.abs(got - ref)) <= 1e-14
 
 
-@pytest.mark.parametrize("name", ["box2d9p", "box2d49p", "box3d27p", "1d5p", "star2d13p"])
+@pytest.mark.parametrize("name", ["box2d9p", "box2d49p", "box3d27p", "1d5p", "star2d13p", "box3d125p",
+                                  "star3d19p"])
 def test_fourier_decay_symbol(name):
     """Centro-symmetric w: lambda(k) = sum_o w_o cos(2 pi k.o/N) (the stencil's symbol)."""
     s = synth.SHAPES[name]

@@ -314,9 +314,13 @@ def test_run_argument_validation_without_gpu():
     assert lib.csx_run(h, None, vp(0x10000), 1, None) == csx.CSX_ERR_INVALID_ARGUMENT
     assert lib.csx_run(h, vp(0x10001), vp(0x90000), 1, None) == csx.CSX_ERR_INVALID_ARGUMENT  # misaligned
     assert lib.csx_run(h, vp(0x10000), vp(0x10000 + 8 * (n // 2)), 1, None) == csx.CSX_ERR_INVALID_ARGUMENT  # overlap
+    assert "overlap" in csx._lib.csx_last_error().decode()
     assert lib.csx_run(h, vp(0x10000), vp(0x90000), -1, None) == csx.CSX_ERR_INVALID_ARGUMENT
+    assert "timesteps" in csx._lib.csx_last_error().decode()
     assert lib.csx_run(None, vp(0x10000), vp(0x90000), 1, None) == csx.CSX_ERR_INVALID_ARGUMENT
-    assert "overlap" in csx._lib.csx_last_error().decode() or True
+    assert "NULL" in csx._lib.csx_last_error().decode()
+    assert lib.csx_plan_set_max_ctas(h, -1) == csx.CSX_ERR_INVALID_ARGUMENT
+    assert lib.csx_plan_set_max_ctas(h, 3) == csx.CSX_OK
     p.close()
 
 

@@ -31,7 +31,8 @@ def test_points_match_paper_names():
     # Table 4 (P.1848-1859): point counts are part of the shape names.
     pts = {n: s.points for n, s in synth.SHAPES.items()}
     assert pts == {"heat1d": 3, "1d5p": 5, "heat2d": 5, "box2d9p": 9, "star2d13p": 13,
-                   "box2d49p": 49, "heat3d": 7, "box3d27p": 27, "star2d9p": 9, "box2d25p": 25}
+                   "box2d49p": 49, "heat3d": 7, "box3d27p": 27, "star2d9p": 9, "box2d25p": 25,
+                   "star3d13p": 13, "box3d125p": 125, "star3d19p": 19, "box3d343p": 343}
 
 
 def test_grid_window_and_torch_generator_match_grid():
