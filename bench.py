@@ -540,6 +540,23 @@ def main():
             roof["tc_share_of_step"] = tc_ms / ms_total if ms_total > 0 else None
             roof["timing"] = "CUDA events around sampled launches inside the timed steps"
         roof["timed_every"] = args.prof_every
+        # hardware counters of the same kernel from the committed ncu pass (scripts/dmma_counters.py:
+        # one main-pass launch of this config and engine): DMMA instructions executed vs the count
+        # the planner states, DMMA-pipe active %, DRAM bytes vs algorithmic
+        hw = (load_json(os.path.join(ROOT, "profiles", "dmma_counters.json")) or {}).get(key)
+        if hw:
+            roof["ncu"] = {
+                "kernel": hw.get("kernel"),
+                "dmma_inst_per_launch": hw.get("sm__inst_executed_pipe_tensor_subpipe_dmma.sum"),
+                "dmma_inst_planner": (hw.get("info") or {}).get("mma_per_pass"),
+                "dmma_inst_vs_planner": hw.get("dmma_inst_vs_planner"),
+                "dmma_pipe_active_pct": hw.get(
+                    "sm__pipe_tensor_subpipe_dmma_cycles_active.avg.pct_of_peak_sustained_elapsed"),
+                "fp64_shared_pipe_active_pct": hw.get(
+                    "sm__pipe_shared_cycles_active.avg.pct_of_peak_sustained_elapsed"),
+                "dram_bytes_per_launch": hw.get("dram_bytes"),
+                "dram_vs_algorithmic": hw.get("dram_vs_algorithmic"),
+                "source": "profiles/dmma_counters.json (ncu --metrics, one main-pass launch, cold L2)"}
 
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
@@ -559,20 +576,39 @@ def main():
     line["clocks"] = clocks
     if rank == 0 and world == 1 and not args.no_comparator and engine != "direct":
         try:
+            # same protocol as the TC line: warm-up runs, then K timed steps with the same L2
+            # flush between them (small grids) and the same CUDA-graph replay
             plan.set_engine("direct")
-            plan.run(d_in, d_out, T, stream)
+            if graph:
+                plan.set_graph(True)
+            for _ in range(args.warmup):
+                plan.run(d_in, d_out, T, stream)
             torch.cuda.synchronize()
-            e0 = torch.cuda.Event(enable_timing=True)
-            e1 = torch.cuda.Event(enable_timing=True)
-            e0.record(stream)
-            plan.run(d_in, d_out, T, stream)
-            e1.record(stream)
+            cev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                   for _ in range(args.steps)]
+            for e0, e1 in cev:
+                if flush is not None:
+                    flush.fill_(1.0)
+                e0.record(stream)
+                plan.run(d_in, d_out, T, stream)
+                e1.record(stream)
             torch.cuda.synchronize()
-            cms = e0.elapsed_time(e1)
+            cms = sum(e0.elapsed_time(e1) for e0, e1 in cev) / args.steps
+            plan.set_graph(False)
             useful = 2.0 * s.points
+            cval = T * points / (cms * 1e-3) / 1e9
+            fp = load_json(os.path.join(ROOT, "PEAKS_FP64.json")) or {}
+            dfma = fp.get("dfma_tflops_sustained") or fp.get("dfma_tflops") or 37.0
+            hbm_roof = hbm * tfm / 16.0             # GSt/s: 16 B per point per pass of Tf steps
+            dfma_roof = dfma * 1e3 / useful          # GSt/s: useful DFMA flops only (no recompute)
             line["comparator"] = {"engine": "direct (CUDA-core DFMA, temporal blocking)",
-                                  "value": T * points / (cms * 1e-3) / 1e9, "unit": UNIT,
-                                  "useful_flops_per_point_step": useful}
+                                  "value": cval, "unit": UNIT, "ms_per_step": cms,
+                                  "useful_flops_per_point_step": useful, "fuse_steps": tfm,
+                                  "roof_gsts": min(hbm_roof, dfma_roof),
+                                  "roof": "hbm" if hbm_roof < dfma_roof else "dfma",
+                                  "frac": cval / min(hbm_roof, dfma_roof),
+                                  "hbm_roof_gsts": hbm_roof, "dfma_roof_gsts": dfma_roof,
+                                  "dfma_peak_tflops": dfma}
             plan.set_engine(args.engine)
         except Exception as e:  # report, do not hide
             line["comparator"] = {"error": str(e)}

@@ -1000,10 +1000,15 @@ using Tile3D3c = Tile3DCfg<3, 8, 2, 4, 6, 32>;     // CTA 64 x 64 outputs, 8 DMM
 using Tile3D3d = Tile3DCfg<3, 2, 8, 1, 5, 32, 2>;  // CTA 64 x 32, 8 warps of 2 block rows x 2 column groups
 using Tile3D3k = Tile3DCfg<3, 8, 2, 2, 5, 32, 1, 1>;  // Tile3D3, k-slice-outer DMMA order
 using Tile3D3ck = Tile3DCfg<3, 8, 2, 4, 6, 32, 1, 1>;  // Tile3D3c, k-slice-outer DMMA order
-// radius 2: 2x4 blocks (K = 6 x 8), 8 DMMA warps, CTA 32 x 64, 6-plane ring, weights per plane
-using Tile3D5 = Tile3DCfg<5, 4, 4, 2, 6, 32, 1, 0, 2, 4, 0>;
-// radius 3: 4x2 blocks (K = 10 x 8), 8 DMMA warps, CTA 32 x 64, 8-plane ring, weights per plane
-using Tile3D7 = Tile3DCfg<7, 4, 2, 4, 8, 32, 1, 0, 4, 2, 0>;
+// wide tiles (the lateral x halo costs a 64-B DRAM granule on each side of every staged row:
+// 25 % extra reads at 64 columns, 12.5 % at 128; the TMA box is <= 256 wide): CTA 32 x 128
+// (8 warps of 2 column groups), 6-plane ring, 32- or 64-plane z chunks
+using Tile3D3w = Tile3DCfg<3, 4, 2, 4, 6, 32, 2, 1>;
+using Tile3D3y = Tile3DCfg<3, 4, 2, 4, 6, 64, 2, 1>;
+// radius 2: 2x4 blocks (K = 6 x 8), 8 DMMA warps, CTA 32 x 64, 9-plane ring (4 planes in flight), weights per plane
+using Tile3D5 = Tile3DCfg<5, 4, 4, 2, 9, 32, 1, 0, 2, 4, 0>;
+// radius 3: 4x2 blocks (K = 10 x 8), 8 DMMA warps, CTA 32 x 64, 10-plane ring (3 in flight), weights per plane
+using Tile3D7 = Tile3DCfg<7, 4, 2, 4, 10, 32, 1, 0, 4, 2, 0>;
 
 
 // ------------------------------------------------------------------------------------------
@@ -1306,6 +1311,8 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
       if (e && e[0] == '0') return launch_tile3d_cfg<Tile3D3>(a, a.tc_mask, st);
       if (e && e[0] == '8') return launch_tile3d_cfg<Tile3D3k>(a, a.tc_mask, st);
       if (e && e[0] == '9') return launch_tile3d_cfg<Tile3D3ck>(a, a.tc_mask, st);
+      if (e && e[0] == '4') return launch_tile3d_cfg<Tile3D3w>(a, a.tc_mask, st);
+      if (e && e[0] == '6') return launch_tile3d_cfg<Tile3D3y>(a, a.tc_mask, st);
       // default: star shapes (one TC plane, HBM-bound) take the 64 x 64 tile with 8 DMMA warps
       // (less halo per plane); box shapes (DMMA-bound) the 64 x 32 tile at 2 CTAs / SM
       // (measured)

@@ -286,7 +286,7 @@ def test_parity_3d_two_step_blocking(csx, name, bc):
         del os.environ["CSX_FORCE_OVERLAP"]
 
 
-@pytest.mark.parametrize("variant", ["0", "1", "2", "3", "8", "9"])
+@pytest.mark.parametrize("variant", ["0", "1", "2", "3", "4", "6", "8", "9"])
 def test_parity_3d_tile_variants(csx, monkeypatch, variant):
     """Every TC_TILE 3D CTA geometry / DMMA order (CSX_TILE3D_VARIANT), star and box, ragged
     (y, x) tiles and z chunks, both boundaries."""
@@ -314,13 +314,17 @@ def test_parity_3d_zchunks(csx, name, engine):
 
 
 def test_direct_comparator_2d_all_radii(csx):
-    """The 2D CUDA-core comparator (k_direct2d) for r = 1..3 and its temporal-blocking depths."""
-    for ndim, r, tf in [(2, 1, 1), (2, 1, 2), (2, 1, 3), (2, 2, 1), (2, 3, 1), (2, 3, 2)]:
+    """The 2D CUDA-core comparator (k_direct2d_wf for r = 1 (Tf <= 4) and r = 2 (Tf = 1), the
+    shared-memory kernels otherwise) for r = 1..3 and its temporal-blocking depths; the second
+    grid spans several 256-row chunks and 56-64-column strips with ragged tails."""
+    for ndim, r, tf in [(2, 1, 1), (2, 1, 2), (2, 1, 3), (2, 1, 4), (2, 2, 1), (2, 2, 2), (2, 3, 1),
+                        (2, 3, 2)]:
         w = synth.random_signed_weights(ndim, r, seed=40 + r)
-        u0 = synth.grid((131, 150), seed=41)
-        for bc in ("fixed", "periodic"):
-            got, info = run_gpu(csx, u0, w, "box", bc, 9, engine="direct", fuse_steps=tf)
-            assert rel(got, oracle.run(u0, w, bc, 9)) <= TOL, (r, tf, bc)
+        for ext in ((131, 150), (601, 333)):
+            u0 = synth.grid(ext, seed=41)
+            for bc in ("fixed", "periodic"):
+                got, info = run_gpu(csx, u0, w, "box", bc, 9, engine="direct", fuse_steps=tf)
+                assert rel(got, oracle.run(u0, w, bc, 9)) <= TOL, (r, tf, bc, ext)
 
 
 @pytest.mark.parametrize("generic", [False, True])
@@ -536,6 +540,45 @@ for r, tf, n, T in [(1, 1, 9001, 13), (1, 11, 20000, 25), (2, 5, 7777, 12), (3, 
         p.close()
 print(worst)
 """
+
+
+_D2_VARIANT_SCRIPT = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+import oracle, synth
+import paper_conf_ppopp_chenlwbwmyzcy24_b200 as csx
+worst = 0.0
+for r, tf in [(1, 1), (1, 2), (1, 3), (1, 4), (2, 1), (2, 2), (3, 1)]:
+    w = synth.random_signed_weights(2, r, seed=40 + r)
+    u0 = synth.grid((601, 333), seed=41)
+    for bc in ("fixed", "periodic"):
+        p = csx.Plan(u0.shape, w, shape="box", bc=bc, fuse_steps=tf, engine="direct")
+        d_in = torch.from_numpy(u0).cuda()
+        d_out = torch.empty_like(d_in)
+        p.run(d_in, d_out, 9)
+        torch.cuda.synchronize()
+        ref = oracle.run(u0, w, bc, 9)
+        worst = max(worst, float(np.max(np.abs(d_out.cpu().numpy() - ref)) / np.max(np.abs(ref))))
+        p.close()
+print(worst)
+"""
+
+
+@pytest.mark.parametrize("env", [{"CSX_DIRECT2D": "smem"}, {"CSX_DIRECT2D": "smem", "CSX_DIRECT_WS": "0"},
+                                 {"CSX_DIRECT2D_V": "4"}, {"CSX_DIRECT2D_UNR": "1"}])
+def test_direct_comparator_2d_variants(env):
+    """Every 2D comparator kernel variant (register wavefront V = 2 / 4, row loop unrolled by 2R+1 or
+    not, the
+    shared-memory kernels with and without warp specialisation; knobs read once per process,
+    hence a subprocess each) matches the oracle."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, "-c", _D2_VARIANT_SCRIPT, root], env=dict(os.environ, **env),
+                         cwd=root, capture_output=True, text=True, timeout=300)
+    assert out.returncode == 0, out.stderr[-2000:]
+    assert float(out.stdout.strip().splitlines()[-1]) <= TOL, (env, out.stdout)
 
 
 @pytest.mark.parametrize("v,pf", [(4, 0), (4, 1), (8, 1), (16, 0), (16, 1), (32, 0)])
