@@ -578,11 +578,13 @@ def main():
         try:
             # same protocol as the TC line: warm-up runs, then K timed steps with the same L2
             # flush between them (small grids) and the same CUDA-graph replay
-            plan.set_engine("direct")
+            # the comparator at ITS OWN best fusion depth (csx_auto_fuse_steps for DIRECT)
+            cplan = csx.Plan(gext, w, shape=s.kind, bc=bc, engine="direct")
+            ctf = cplan.info()["fuse_steps"]
             if graph:
-                plan.set_graph(True)
+                cplan.set_graph(True)
             for _ in range(args.warmup):
-                plan.run(d_in, d_out, T, stream)
+                cplan.run(d_in, d_out, T, stream)
             torch.cuda.synchronize()
             cev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
                    for _ in range(args.steps)]
@@ -590,26 +592,25 @@ def main():
                 if flush is not None:
                     flush.fill_(1.0)
                 e0.record(stream)
-                plan.run(d_in, d_out, T, stream)
+                cplan.run(d_in, d_out, T, stream)
                 e1.record(stream)
             torch.cuda.synchronize()
             cms = sum(e0.elapsed_time(e1) for e0, e1 in cev) / args.steps
-            plan.set_graph(False)
+            cplan.close()
             useful = 2.0 * s.points
             cval = T * points / (cms * 1e-3) / 1e9
             fp = load_json(os.path.join(ROOT, "PEAKS_FP64.json")) or {}
             dfma = fp.get("dfma_tflops_sustained") or fp.get("dfma_tflops") or 37.0
-            hbm_roof = hbm * tfm / 16.0             # GSt/s: 16 B per point per pass of Tf steps
+            hbm_roof = hbm * ctf / 16.0             # GSt/s: 16 B per point per pass of Tf steps
             dfma_roof = dfma * 1e3 / useful          # GSt/s: useful DFMA flops only (no recompute)
             line["comparator"] = {"engine": "direct (CUDA-core DFMA, temporal blocking)",
                                   "value": cval, "unit": UNIT, "ms_per_step": cms,
-                                  "useful_flops_per_point_step": useful, "fuse_steps": tfm,
+                                  "useful_flops_per_point_step": useful, "fuse_steps": ctf,
                                   "roof_gsts": min(hbm_roof, dfma_roof),
                                   "roof": "hbm" if hbm_roof < dfma_roof else "dfma",
                                   "frac": cval / min(hbm_roof, dfma_roof),
                                   "hbm_roof_gsts": hbm_roof, "dfma_roof_gsts": dfma_roof,
                                   "dfma_peak_tflops": dfma}
-            plan.set_engine(args.engine)
         except Exception as e:  # report, do not hide
             line["comparator"] = {"error": str(e)}
     if not args.no_e2e:

@@ -102,7 +102,7 @@ cudaError_t launch_direct(const DirectArgs& a, cudaStream_t st);
 // 2D comparator kernel (kernels_direct2d.cu): compile-time (r, Tf), weights by value.
 bool direct2d_exists(int r, int tf);
 // register-wavefront 2D comparator (kernels_direct2d_wf.cu): R = 1 (Tf <= 4), 2 (Tf <= 2), 3 (Tf = 1)
-bool direct2d_wf_exists(int r, int tf);
+bool direct2d_wf_exists(int r, int tf, const double* w_host);
 cudaError_t launch_direct2d_wf(const DirectArgs& a, const double* w_host, cudaStream_t st);
 cudaError_t launch_direct2d(const DirectArgs& a, const double* w_host, cudaStream_t st);
 // 1D / 3D comparator kernels (kernels_direct13.cu): compile-time r, weights by value.

@@ -400,17 +400,17 @@ bool direct2d_exists(int r, int tf) {
 
 // which 2D comparator kernel: CSX_DIRECT2D=wf (default: register wavefront, where it exists) or
 // smem (the shared-memory temporal-blocking kernels below; CSX_DIRECT_WS picks ws / plain)
-static bool use_wf(int r, int tf) {
+static bool use_wf(int r, int tf, const double* w) {
   static const int smem = [] {
     const char* e = getenv("CSX_DIRECT2D");
     return e && e[0] == 's';
   }();
-  return !smem && direct2d_wf_exists(r, tf);
+  return !smem && direct2d_wf_exists(r, tf, w);
 }
 
 // The base weights travel by value as kernel parameters (constant-bank DFMA operands).
 cudaError_t launch_direct2d(const DirectArgs& a, const double* w_host, cudaStream_t st) {
-  if (use_wf(a.r, a.tf)) {
+  if (use_wf(a.r, a.tf, w_host)) {
     const cudaError_t e = launch_direct2d_wf(a, w_host, st);
     if (e != cudaErrorNotSupported) return e;
   }

@@ -80,7 +80,7 @@ __device__ __forceinline__ void wf_extend(const double* o, double* e) {
   }
 }
 
-template <int R, int TF, int V, int UNR, bool EDGE>
+template <int R, int TF, int V, int UNR, bool STAR, bool EDGE>
 __device__ __forceinline__ void wf_item(const DirectArgs& a, const WFWeights& Wt, double* ring, int64_t r0,
                                         int64_t r1, int64_t x0, int64_t xs0, int64_t xs1, int lane) {
   using C = WFCfg<R, TF, V>;
@@ -164,6 +164,7 @@ __device__ __forceinline__ void wf_item(const DirectArgs& a, const WFWeights& Wt
         for (int k = 0; k < N; ++k)
 #pragma unroll
           for (int b = 0; b < N; ++b) {
+            if (STAR && k != R && b != R) continue;  // star footprint: axial taps only
             const double xv = win[l - 1][k][q + b];
             if ((k * N + b) & 1) v1 = fma(Wt.w[k * N + b], xv, v1);
             else v0 = fma(Wt.w[k * N + b], xv, v0);
@@ -204,7 +205,7 @@ __device__ __forceinline__ void wf_item(const DirectArgs& a, const WFWeights& Wt
   __syncwarp();
 }
 
-template <int R, int TF, int V, int BH, int UNR>
+template <int R, int TF, int V, int BH, int UNR, bool STAR>
 __global__ void __launch_bounds__(128) k_direct2d_wf(DirectArgs a, WFWeights Wt) {
   using C = WFCfg<R, TF, V>;
   extern __shared__ __align__(16) double wf_smem[];
@@ -226,13 +227,13 @@ __global__ void __launch_bounds__(128) k_direct2d_wf(DirectArgs a, WFWeights Wt)
       const int64_t gx0 = x0 + a.gorg[2], gx1 = x0 + C::W + a.gorg[2];
       edge = gy0 < R || gy1 > a.GE[1] - R || gx0 < R || gx1 > a.GE[2] - R;
     }
-    if (edge) wf_item<R, TF, V, UNR, true>(a, Wt, ring, r0, r1, x0, xs0, xs1, lane);
-    else wf_item<R, TF, V, UNR, false>(a, Wt, ring, r0, r1, x0, xs0, xs1, lane);
+    if (edge) wf_item<R, TF, V, UNR, STAR, true>(a, Wt, ring, r0, r1, x0, xs0, xs1, lane);
+    else wf_item<R, TF, V, UNR, STAR, false>(a, Wt, ring, r0, r1, x0, xs0, xs1, lane);
   }
 }
 
-template <int R, int TF, int V, int UNR = 1>
-static cudaError_t launch_wf(const DirectArgs& a, const double* w_host, cudaStream_t st) {
+template <int R, int TF, int V, int UNR, bool STAR>
+static cudaError_t launch_wf_s(const DirectArgs& a, const double* w_host, cudaStream_t st) {
   using C = WFCfg<R, TF, V>;
   constexpr int BH = 256;
   // the row loop reads up to 2N rows past the chunk's last halo row and the strip's columns
@@ -242,16 +243,31 @@ static cudaError_t launch_wf(const DirectArgs& a, const double* w_host, cudaStre
   const int n = 2 * R + 1;
   for (int i = 0; i < 49; ++i) W.w[i] = i < n * n ? w_host[i] : 0.0;
   int occ = 0;
-  cudaError_t e = cudaFuncSetAttribute(k_direct2d_wf<R, TF, V, BH, UNR>,
+  cudaError_t e = cudaFuncSetAttribute(k_direct2d_wf<R, TF, V, BH, UNR, STAR>,
                                        cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
   if (e != cudaSuccess) return e;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_direct2d_wf<R, TF, V, BH, UNR>, C::NT, C::SMEM);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_direct2d_wf<R, TF, V, BH, UNR, STAR>, C::NT, C::SMEM);
   if (e != cudaSuccess) return e;
   const int64_t items = ((a.E[2] + C::S - 1) / C::S) * ((a.E[1] + BH - 1) / BH);
   const int64_t grid = persistent_grid(occ, a.max_ctas, (items + 3) / 4);
   if (grid < 1) return cudaSuccess;
-  k_direct2d_wf<R, TF, V, BH, UNR><<<(unsigned)grid, C::NT, C::SMEM, st>>>(a, W);
+  k_direct2d_wf<R, TF, V, BH, UNR, STAR><<<(unsigned)grid, C::NT, C::SMEM, st>>>(a, W);
   return cudaGetLastError();
+}
+
+// star weights (every off-axis tap zero): the kernel skips those taps at compile time
+static bool wf_star(int r, const double* w) {
+  const int n = 2 * r + 1;
+  for (int k = 0; k < n; ++k)
+    for (int b = 0; b < n; ++b)
+      if (k != r && b != r && w[k * n + b] != 0.0) return false;
+  return true;
+}
+
+template <int R, int TF, int V, int UNR = 1>
+static cudaError_t launch_wf(const DirectArgs& a, const double* w_host, cudaStream_t st) {
+  return wf_star(R, w_host) ? launch_wf_s<R, TF, V, UNR, true>(a, w_host, st)
+                            : launch_wf_s<R, TF, V, UNR, false>(a, w_host, st);
 }
 
 static int wf_v() {
@@ -272,10 +288,14 @@ static int wf_unr() {
   return v;
 }
 
-// (R = 3, Tf = 2 holds 2 x 7 x 8 window doubles per lane and spills: it keeps the shared-memory
-// kernel of kernels_direct2d.cu; V = 4 only up to Tf = 2)
-bool direct2d_wf_exists(int r, int tf) {
-  return (r == 1 && tf >= 1 && tf <= 4) || (r == 2 && tf <= 2) || (r == 3 && tf == 1);
+// Where the register window is larger than the shared-memory kernels' working set (box r = 2,
+// Tf = 2: 2 x 5 x 6 doubles per lane; box r = 3: 7 x 8, spilling) those kernels measured faster
+// (240 vs 223, 151 vs 139 GSt/s on B200) and keep the case; star weights skip most taps here.
+// (r = 3, Tf = 2 spills outright; V = 4 only up to Tf = 2)
+bool direct2d_wf_exists(int r, int tf, const double* w) {
+  const bool star = wf_star(r, w);
+  return (r == 1 && tf >= 1 && tf <= 4) || (r == 2 && tf == 1) || (r == 2 && tf == 2 && star) ||
+         (r == 3 && tf == 1 && star);
 }
 
 cudaError_t launch_direct2d_wf(const DirectArgs& a, const double* w_host, cudaStream_t st) {

@@ -15,6 +15,8 @@
 //       (star arms) on CUDA cores in the same kernel (P.1788-1800).
 #include <cuda_runtime.h>
 
+#include <cstdlib>
+
 #include "kernels.cuh"
 #include "s2r_geom.h"
 
@@ -190,6 +192,143 @@ __global__ void __launch_bounds__(S2R2D<NK>::NT, 2) k_s2r2d(S2RArgs a) {
         }
       }
     }
+#pragma unroll
+    for (int q = 0; q < RW; ++q) {
+      const int64_t row = (int64_t)ty * G::BM + xr0 + q;
+      if (row < a.E1) store_pair(a.dst.p + row * a.dst.s1, col, a.E2, v0, v1, c[q][0], c[q][1]);
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+// 2D, warp-specialised (the default for the DMMA variants III / IV / V): the LUT scatter and the
+// dual tessellation run on DIFFERENT warps, so the DMMA warps never wait for a scatter.
+//   warp NCW + NSW      producer: raw input regions -> RAW_STAGES ring (cp.async.bulk rows)
+//   warps NCW .. +NSW   scatter: raw stage -> stencil2row A/B buffer it % 2 through the LUT
+//   warps 0 .. NCW-1    dual tessellation on DMMA from A/B buffer it % 2, centre store
+// Buffer hand-offs are mbarriers: raw full/empty, ab_full (scatter warps arrive) and ab_empty
+// (DMMA warps arrive), so tile k+1 is scattered while tile k is tessellated.
+template <int NK, bool PAD = true>
+struct S2R2DWS {
+  using G = S2R2D<NK, PAD>;
+  // nk = 7 keeps 26 weight fragments per DMMA lane: at 2 CTAs / SM two scatter warps make the
+  // DMMA warps spill (80 registers: 0.646 of the DMMA roof) and one cannot keep up (0.447), so
+  // nk = 7 runs one CTA per SM with four scatter warps and a 2-stage raw ring; nk <= 5 runs two
+  // CTAs per SM with two scatter warps
+  static constexpr int MINB = NK >= 7 ? 1 : 2;
+  static constexpr int NSW = NK >= 7 ? 4 : 2;
+  static constexpr int RAW_STAGES = 2;
+  static constexpr int NT = 32 * (G::NCW + NSW + 1);
+  static constexpr int SMEM = RAW_STAGES * G::RAW * 8 + G::AB_BUFS * G::AB * 8 + G::NE * 4;
+};
+
+template <int NK, bool PAD, bool DIRTY>
+__global__ void __launch_bounds__(S2R2DWS<NK>::NT, S2R2DWS<NK>::MINB) k_s2r2d_ws(S2RArgs a) {
+  using G = S2R2D<NK, PAD>;
+  using W = S2R2DWS<NK, PAD>;
+  constexpr int NSW = W::NSW;
+  extern __shared__ __align__(128) double smem[];
+  __shared__ __align__(8) uint64_t full[W::RAW_STAGES], empty[W::RAW_STAGES], ab_full[2], ab_empty[2];
+  double* raw = smem;                                           // RAW_STAGES x RAW
+  double* sAB = raw + W::RAW_STAGES * G::RAW;                   // 2 x (A | B)
+  uint32_t* sL = reinterpret_cast<uint32_t*>(sAB + G::AB_BUFS * G::AB);
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  for (int i = tid; i < G::AB_BUFS * G::AB; i += S2R2DWS<NK>::NT) sAB[i] = 0.0;
+  for (int i = tid; i < G::NE; i += S2R2DWS<NK>::NT) sL[i] = (uint32_t)a.lut[i].y;
+  if (tid == 0) {
+    for (int s = 0; s < W::RAW_STAGES; ++s) {
+      s2r_mbar_init(&full[s], 1);
+      s2r_mbar_init(&empty[s], NSW);
+    }
+    for (int b = 0; b < 2; ++b) {
+      s2r_mbar_init(&ab_full[b], NSW);
+      s2r_mbar_init(&ab_empty[b], G::NCW);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  __syncthreads();
+  if (warp == G::NCW + NSW) {  // producer
+    int it = 0;
+    for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
+      const int s = it % W::RAW_STAGES, n = it / W::RAW_STAGES;
+      if (n > 0) s2r_mbar_wait(&empty[s], (n - 1) & 1);
+      const int ty = (int)(tile / a.tiles_x);
+      const int tx = (int)(tile - (int64_t)ty * a.tiles_x);
+      const double* src = a.src.p + (int64_t)(ty * G::BM - G::R) * a.src.s1 + (tx * G::BN - G::R - G::ODD);
+      s2r_issue_rows(src, a.src.s1, raw + s * G::RAW, G::RR, G::TPR, &full[s], lane);
+    }
+    return;
+  }
+  if (warp >= G::NCW) {  // scatter warps: implicit stencil2row through the LUT (branch-free)
+    const int sw = warp - G::NCW;
+    int it = 0;
+    for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
+      const int s = it % W::RAW_STAGES, b = it & 1;
+      if (it >= 2) s2r_mbar_wait(&ab_empty[b], ((it >> 1) - 1) & 1);  // tile it-2 tessellated
+      s2r_mbar_wait(&full[s], (it / W::RAW_STAGES) & 1);
+      double* sA = sAB + b * G::AB;
+      double* sB = sA + (G::STRIPS + 1) * G::PITCH;
+      const double* rs = raw + s * G::RAW + G::ODD;
+      for (int x = sw; x < G::RR; x += NSW) {
+        const double* rrow = rs + x * G::TPR;
+        const uint32_t* lrow = sL + x * G::RC;
+        for (int y = lane; y < G::RC; y += 32) {
+          const double v = rrow[y];
+          const uint32_t l = lrow[y];
+          if (DIRTY) {  // dirty bits absorb the unused elements: no branch (P.1759-1773)
+            sA[l & 0xffffu] = v;
+            sB[l >> 16] = v;
+          } else {      // breakdown variants III / IV: conditional stores
+            if ((l & 0xffffu) != 0xffffu) sA[l & 0xffffu] = v;
+            if ((l >> 16) != 0xffffu) sB[l >> 16] = v;
+          }
+        }
+      }
+      __syncwarp();
+      if (lane == 0) {
+        s2r_mbar_arrive(&empty[s]);    // raw stage consumed
+        s2r_mbar_arrive(&ab_full[b]);  // this warp's share of A/B written
+      }
+    }
+    return;
+  }
+  // DMMA warps
+  double wa[G::KS], wb[G::KS];
+#pragma unroll
+  for (int s = 0; s < G::KS; ++s) {
+    wa[s] = a.frags[s * 32 + lane];
+    wb[s] = a.frags[(G::KS + s) * 32 + lane];
+  }
+  const int g = lane >> 2, t = lane & 3;
+  const bool v0 = 2 * t < G::SW, v1 = 2 * t + 1 < G::SW;
+  constexpr int RW = G::BM / G::NCW;
+  const int xr0 = warp * RW;
+  int it = 0;
+  for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
+    const int b = it & 1;
+    const int ty = (int)(tile / a.tiles_x);
+    const int tx = (int)(tile - (int64_t)ty * a.tiles_x);
+    s2r_mbar_wait(&ab_full[b], (it >> 1) & 1);
+    const double* sA = sAB + b * G::AB;
+    const double* sB = sA + (G::STRIPS + 1) * G::PITCH;
+    const double* pa = sA + g * G::PITCH + G::NKV * xr0 + t;
+    const double* pb = sB + g * G::PITCH + G::NKV * xr0 + t;
+    double c[RW][2];
+#pragma unroll
+    for (int q = 0; q < RW; ++q) c[q][0] = c[q][1] = 0.0;
+    // the warp's RW output rows as RW independent chains, vitrolite B accumulated onto A
+    // (P.1332-1336)
+#pragma unroll
+    for (int s2 = 0; s2 < G::KS; ++s2)
+#pragma unroll
+      for (int q = 0; q < RW; ++q) dmma(c[q][0], c[q][1], pa[4 * s2 + q * G::NKV], wa[s2]);
+#pragma unroll
+    for (int s2 = 0; s2 < G::KS; ++s2)
+#pragma unroll
+      for (int q = 0; q < RW; ++q) dmma(c[q][0], c[q][1], pb[4 * s2 + q * G::NKV], wb[s2]);
+    __syncwarp();
+    if (lane == 0) s2r_mbar_arrive(&ab_empty[b]);  // A/B buffer b no longer read by this warp
+    const int64_t col = (int64_t)tx * G::BN + g * G::SW + 2 * t;
 #pragma unroll
     for (int q = 0; q < RW; ++q) {
       const int64_t row = (int64_t)ty * G::BM + xr0 + q;
@@ -397,12 +536,30 @@ static cudaError_t launch_persistent(K kernel, int smem, int nthreads, int64_t i
   return cudaGetLastError();
 }
 
+// CSX_S2R_WS=0 selects the round-1 kernel (scatter and tessellation on the same 8 warps)
+static bool s2r_ws() {
+  static const int v = [] {
+    const char* e = getenv("CSX_S2R_WS");
+    return e ? atoi(e) : 1;
+  }();
+  return v != 0;
+}
+
 template <int NK>
 static cudaError_t launch_s2r2d_var(const S2RArgs& a, int variant, cudaStream_t st) {
   // variant bit 0 = padding, bit 1 = dirty bits (default 3 = the paper's full design),
   // bit 2 = CUDA-core tessellation (breakdown II, with padding and dirty bits)
   if (variant & 4)
     return launch_persistent(k_s2r2d<NK, true, true, true>, S2R2D<NK, true>::SMEM, S2R2D<NK>::NT, a.ntiles, st, a);
+  if (s2r_ws()) {  // warp-specialised scatter / tessellation (default)
+    constexpr int NT = S2R2DWS<NK>::NT;
+    switch (variant) {
+      case 3: return launch_persistent(k_s2r2d_ws<NK, true, true>, S2R2DWS<NK, true>::SMEM, NT, a.ntiles, st, a);
+      case 1: return launch_persistent(k_s2r2d_ws<NK, true, false>, S2R2DWS<NK, true>::SMEM, NT, a.ntiles, st, a);
+      case 2: return launch_persistent(k_s2r2d_ws<NK, false, true>, S2R2DWS<NK, false>::SMEM, NT, a.ntiles, st, a);
+      default: return launch_persistent(k_s2r2d_ws<NK, false, false>, S2R2DWS<NK, false>::SMEM, NT, a.ntiles, st, a);
+    }
+  }
   switch (variant) {
     case 3: return launch_persistent(k_s2r2d<NK, true, true>, S2R2D<NK, true>::SMEM, S2R2D<NK>::NT, a.ntiles, st, a);
     case 1: return launch_persistent(k_s2r2d<NK, true, false>, S2R2D<NK, true>::SMEM, S2R2D<NK>::NT, a.ntiles, st, a);

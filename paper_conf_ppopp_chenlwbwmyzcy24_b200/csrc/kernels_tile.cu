@@ -1005,6 +1005,10 @@ using Tile3D3ck = Tile3DCfg<3, 8, 2, 4, 6, 32, 1, 1>;  // Tile3D3c, k-slice-oute
 // (8 warps of 2 column groups), 6-plane ring, 32- or 64-plane z chunks
 using Tile3D3w = Tile3DCfg<3, 4, 2, 4, 6, 32, 2, 1>;
 using Tile3D3y = Tile3DCfg<3, 4, 2, 4, 6, 64, 2, 1>;
+// long z runs (the z-chunk halo planes are re-read from DRAM: 2 / ZCH extra): 64 x 64 tiles with
+// 128-plane chunks (1 CTA / SM), 64 x 32 tiles with 256-plane chunks (2 CTAs / SM)
+using Tile3D3z = Tile3DCfg<3, 8, 2, 4, 6, 128, 1, 1>;
+using Tile3D3l = Tile3DCfg<3, 8, 2, 2, 5, 256, 1, 1>;
 // radius 2: 2x4 blocks (K = 6 x 8), 8 DMMA warps, CTA 32 x 64, 9-plane ring (4 planes in flight), weights per plane
 using Tile3D5 = Tile3DCfg<5, 4, 4, 2, 9, 32, 1, 0, 2, 4, 0>;
 // radius 3: 4x2 blocks (K = 10 x 8), 8 DMMA warps, CTA 32 x 64, 10-plane ring (3 in flight), weights per plane
@@ -1313,6 +1317,8 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
       if (e && e[0] == '9') return launch_tile3d_cfg<Tile3D3ck>(a, a.tc_mask, st);
       if (e && e[0] == '4') return launch_tile3d_cfg<Tile3D3w>(a, a.tc_mask, st);
       if (e && e[0] == '6') return launch_tile3d_cfg<Tile3D3y>(a, a.tc_mask, st);
+      if (e && e[0] == '5') return launch_tile3d_cfg<Tile3D3z>(a, a.tc_mask, st);
+      if (e && e[0] == '7') return launch_tile3d_cfg<Tile3D3l>(a, a.tc_mask, st);
       // default: star shapes (one TC plane, HBM-bound) take the 64 x 64 tile with 8 DMMA warps
       // (less halo per plane); box shapes (DMMA-bound) the 64 x 32 tile at 2 CTAs / SM
       // (measured)

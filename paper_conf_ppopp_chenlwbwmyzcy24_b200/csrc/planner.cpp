@@ -336,6 +336,9 @@ int auto_tf(int ndim, int radius, int engine) {
     if (engine == CSX_ENGINE_TC_S2R) return radius == 1 ? 7 : (radius == 2 ? 3 : 2);
     return radius == 1 ? 11 : (radius == 2 ? 5 : 3);
   }
+  // the CUDA-core comparator's own best depth: 2D r = 1 -> 4 (register wavefront, Box-2D9P
+  // 10240^2: Tf 1/2/3/4 = 310 / 640 / 681 / 766 GSt/s), r >= 2 -> 1
+  if (ndim == 2 && engine == CSX_ENGINE_DIRECT) return radius == 1 ? 4 : 1;
   if (ndim == 2) return radius == 1 ? 3 : 1;
   return 1;
 }

@@ -286,7 +286,7 @@ def test_parity_3d_two_step_blocking(csx, name, bc):
         del os.environ["CSX_FORCE_OVERLAP"]
 
 
-@pytest.mark.parametrize("variant", ["0", "1", "2", "3", "4", "6", "8", "9"])
+@pytest.mark.parametrize("variant", ["0", "1", "2", "3", "4", "5", "6", "7", "8", "9"])
 def test_parity_3d_tile_variants(csx, monkeypatch, variant):
     """Every TC_TILE 3D CTA geometry / DMMA order (CSX_TILE3D_VARIANT), star and box, ragged
     (y, x) tiles and z chunks, both boundaries."""
@@ -579,6 +579,47 @@ def test_direct_comparator_2d_variants(env):
                          cwd=root, capture_output=True, text=True, timeout=300)
     assert out.returncode == 0, out.stderr[-2000:]
     assert float(out.stdout.strip().splitlines()[-1]) <= TOL, (env, out.stdout)
+
+
+_S2R_SCRIPT = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+import oracle, synth
+import paper_conf_ppopp_chenlwbwmyzcy24_b200 as csx
+worst = 0.0
+for name in ("box2d9p", "heat2d", "box2d25p", "box2d49p"):
+    s = synth.SHAPES[name]
+    w = synth.random_weights(name)
+    u0 = synth.grid((99, 140), seed=51)
+    for bc in ("fixed", "periodic"):
+        for pad, dirty in ((1, 1), (0, 0), (1, 0), (0, 1)):
+            p = csx.Plan(u0.shape, w, shape=s.kind, bc=bc, engine="tc_s2r")
+            p.set_max_ctas(3)
+            p.set_s2r_variant(bool(pad), bool(dirty))
+            d_in = torch.from_numpy(u0).cuda()
+            d_out = torch.empty_like(d_in)
+            p.run(d_in, d_out, 7)
+            torch.cuda.synchronize()
+            ref = oracle.run(u0, w, bc, 7)
+            worst = max(worst, float(np.max(np.abs(d_out.cpu().numpy() - ref)) / np.max(np.abs(ref))))
+            p.close()
+print(worst)
+"""
+
+
+@pytest.mark.parametrize("ws", ["0", "1"])
+def test_s2r_2d_kernel_variants(ws):
+    """The TC_S2R 2D kernels with the LUT scatter on dedicated warps (CSX_S2R_WS=1, default) and
+    on the tessellation warps (0), every padding / dirty-bits variant, persistent grid capped at 3
+    CTAs so that both A/B buffers and the raw ring wrap many times; read once per process."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, "-c", _S2R_SCRIPT, root], env=dict(os.environ, CSX_S2R_WS=ws),
+                         cwd=root, capture_output=True, text=True, timeout=300)
+    assert out.returncode == 0, out.stderr[-2000:]
+    assert float(out.stdout.strip().splitlines()[-1]) <= TOL, (ws, out.stdout)
 
 
 @pytest.mark.parametrize("v,pf", [(4, 0), (4, 1), (8, 1), (16, 0), (16, 1), (32, 0)])
