@@ -560,7 +560,7 @@ __device__ __forceinline__ void issue_plane(const S2RArgs& a, const CUtensorMap*
 
 __device__ __forceinline__ int ring_next(int s, int n) { return s + 1 == n ? 0 : s + 1; }
 
-template <class C>
+template <class C, bool ONE = false>  // ONE: a single TC plane (star shapes)
 __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
     k_tile3d(S2RArgs a, int tc_mask, const __grid_constant__ CUtensorMap tmap) {
   extern __shared__ __align__(128) double smem_raw[];
@@ -606,6 +606,13 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
 #pragma unroll
       for (int k = 0; k < C::KS; ++k) wf[C::WREG ? p : 0][k] = a.frags[(p * C::KS + k) * 32 + lane];
     wz[p] = a.wc[(p * C::NK + C::R) * C::NK + C::R];
+  }
+  // star shapes have one TC plane (the centre): its fragments stay in registers for the launch
+  constexpr bool single_tc = ONE;
+  if (!C::WREG && single_tc) {
+    const int dz1 = __ffs(tc_mask) - 1;
+#pragma unroll
+    for (int k = 0; k < C::KS; ++k) wf[0][k] = __ldg(a.frags + (dz1 * C::KS + k) * 32 + lane);
   }
   const int alpha = (2 * t) / C::B, beta = (2 * t) % C::B;
   const bool any_cuda = tc_mask != (1 << C::NK) - 1;
@@ -653,7 +660,7 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
 #pragma unroll
       for (int dz = 0; dz < C::NK; ++dz) {
         const double* stg = smem + slot[dz] * C::STAGE_A;
-        if (!C::WREG && (tc_mask & (1 << dz))) {  // this plane's fragments, from L1
+        if (!C::WREG && !single_tc && (tc_mask & (1 << dz))) {  // this plane's fragments, from L1
 #pragma unroll
           for (int k = 0; k < C::KS; ++k) wf[0][k] = __ldg(a.frags + (dz * C::KS + k) * 32 + lane);
         }
@@ -1009,10 +1016,17 @@ using Tile3D3y = Tile3DCfg<3, 4, 2, 4, 6, 64, 2, 1>;
 // 128-plane chunks (1 CTA / SM), 64 x 32 tiles with 256-plane chunks (2 CTAs / SM)
 using Tile3D3z = Tile3DCfg<3, 8, 2, 4, 6, 128, 1, 1>;
 using Tile3D3l = Tile3DCfg<3, 8, 2, 2, 5, 256, 1, 1>;
+// one item per (y, x) tile column: 64 x 64 (1 CTA / SM) or 64 x 32 (2 CTAs / SM) tiles over the
+// whole z extent (no z-chunk halo re-reads; neighbouring columns advance in step)
+using Tile3D3za = Tile3DCfg<3, 8, 2, 4, 6, 1 << 20, 1, 1>;
+using Tile3D3zb = Tile3DCfg<3, 8, 2, 2, 5, 1 << 20, 1, 1>;
 // radius 2: 2x4 blocks (K = 6 x 8), 8 DMMA warps, CTA 32 x 64, 9-plane ring (4 planes in flight), weights per plane
 using Tile3D5 = Tile3DCfg<5, 4, 4, 2, 9, 32, 1, 0, 2, 4, 0>;
 // radius 3: 4x2 blocks (K = 10 x 8), 8 DMMA warps, CTA 32 x 64, 10-plane ring (3 in flight), weights per plane
 using Tile3D7 = Tile3DCfg<7, 4, 2, 4, 10, 32, 1, 0, 4, 2, 0>;
+// the same with the k-slice-outer DMMA order (G independent accumulator chains per k-slice)
+using Tile3D5k = Tile3DCfg<5, 4, 4, 2, 9, 32, 1, 1, 2, 4, 0>;
+using Tile3D7k = Tile3DCfg<7, 4, 2, 4, 10, 32, 1, 1, 4, 2, 0>;
 
 
 // ------------------------------------------------------------------------------------------
@@ -1290,13 +1304,15 @@ static cudaError_t launch_tile3d_cfg(S2RArgs a, int tc_mask, cudaStream_t st) {
   if (a.ntiles == 0) return cudaSuccess;
   CUtensorMap tmap;
   if (!make_tmap(a, C::TP, C::RR, &tmap)) return cudaErrorNotSupported;  // 3D stages by TMA only
-  cudaError_t e = cudaFuncSetAttribute(k_tile3d<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
+  // star shapes (one TC plane) keep that plane's fragments in registers (C::WREG = 0 configs)
+  auto kern = (!C::WREG && __builtin_popcount((unsigned)tc_mask) == 1) ? k_tile3d<C, true> : k_tile3d<C, false>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
   if (e != cudaSuccess) return e;
   int occ = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_tile3d<C>, C::NT, C::SMEM);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, C::NT, C::SMEM);
   if (e != cudaSuccess) return e;
   const int64_t grid = persistent_grid(occ, a.max_ctas, a.ntiles);
-  return launch_pdl(a.pdl != 0, k_tile3d<C>, grid, C::NT, C::SMEM, st, a, tc_mask, tmap);
+  return launch_pdl(a.pdl != 0, kern, grid, C::NT, C::SMEM, st, a, tc_mask, tmap);
 }
 
 cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStream_t st) {
@@ -1305,8 +1321,13 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
   if (ndim == 1) return launch_tile1d(nk, a, st);
   if (ndim == 3) {
     if (tf == 2) return launch_tile3d_tb<Tile3DTB>(a, a.tc_mask, st);  // r = 1: temporal blocking
-    if (nk == 5) return launch_tile3d_cfg<Tile3D5>(a, a.tc_mask, st);
-    if (nk == 7) return launch_tile3d_cfg<Tile3D7>(a, a.tc_mask, st);
+    if (nk == 5 || nk == 7) {
+      // k-slice-outer DMMA order by default (box r = 2 / 3: 56.4 -> 60.0 / 26.6 -> 27.6 GSt/s)
+      const char* e = getenv("CSX_TILE3D_KO");
+      const bool ko = e ? e[0] == '1' : true;
+      if (nk == 5) return ko ? launch_tile3d_cfg<Tile3D5k>(a, a.tc_mask, st) : launch_tile3d_cfg<Tile3D5>(a, a.tc_mask, st);
+      return ko ? launch_tile3d_cfg<Tile3D7k>(a, a.tc_mask, st) : launch_tile3d_cfg<Tile3D7>(a, a.tc_mask, st);
+    }
     if (nk == 3) {
       const char* e = getenv("CSX_TILE3D_VARIANT");
       if (e && e[0] == '1') return launch_tile3d_cfg<Tile3D3b>(a, a.tc_mask, st);
@@ -1319,6 +1340,8 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
       if (e && e[0] == '6') return launch_tile3d_cfg<Tile3D3y>(a, a.tc_mask, st);
       if (e && e[0] == '5') return launch_tile3d_cfg<Tile3D3z>(a, a.tc_mask, st);
       if (e && e[0] == '7') return launch_tile3d_cfg<Tile3D3l>(a, a.tc_mask, st);
+      if (e && e[0] == 'a') return launch_tile3d_cfg<Tile3D3za>(a, a.tc_mask, st);
+      if (e && e[0] == 'b') return launch_tile3d_cfg<Tile3D3zb>(a, a.tc_mask, st);
       // default: star shapes (one TC plane, HBM-bound) take the 64 x 64 tile with 8 DMMA warps
       // (less halo per plane); box shapes (DMMA-bound) the 64 x 32 tile at 2 CTAs / SM
       // (measured)

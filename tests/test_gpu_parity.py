@@ -286,7 +286,7 @@ def test_parity_3d_two_step_blocking(csx, name, bc):
         del os.environ["CSX_FORCE_OVERLAP"]
 
 
-@pytest.mark.parametrize("variant", ["0", "1", "2", "3", "4", "5", "6", "7", "8", "9"])
+@pytest.mark.parametrize("variant", ["0", "1", "2", "3", "4", "5", "6", "7", "8", "9", "a", "b"])
 def test_parity_3d_tile_variants(csx, monkeypatch, variant):
     """Every TC_TILE 3D CTA geometry / DMMA order (CSX_TILE3D_VARIANT), star and box, ragged
     (y, x) tiles and z chunks, both boundaries."""
