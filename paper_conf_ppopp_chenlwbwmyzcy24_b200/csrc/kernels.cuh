@@ -44,6 +44,7 @@ struct S2RArgs {
   int use_tma = 0;                // TC_TILE 2D/3D: stage tiles with one TMA tensor copy
   int l2hint = 0;                 // TMA loads' L2 eviction priority: 0 normal, 1 last, 2 first
   int64_t tma_x0 = 0, tma_y0 = 0, tma_z0 = 0;  // interior origin in tensor-map coordinates
+  int lockstep = 0;               // 3D experiment: producers sync grid-wide every k planes
   int r = 0;
   const double* wbase = nullptr;  // base weights (2r+1)^2
   int64_t gorg0 = 0, gorg1 = 0, gorg2 = 0;  // local origin in global coordinates

@@ -543,6 +543,8 @@ struct Tile3DCfg {
   static_assert(TP <= 256 && RR <= 256, "TMA box dimensions");
 };
 
+__device__ unsigned long long g_lock_ctr[1];  // CSX_LOCKSTEP experiment counter
+
 template <class C>
 __device__ __forceinline__ void issue_plane(const S2RArgs& a, const CUtensorMap* tmap, int ty, int tx,
                                             int64_t zi, double* stage, uint64_t* bar, int lane) {
@@ -580,12 +582,41 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
   if (warp == C::NCW) {  // producer: planes of every work item, in consumption order
     if (lane == 0) tma_prefetch_desc(&tmap);
     int s = 0, round = 0;  // ring slot and how many times the ring has been filled
-    for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
-      const int zcl = (int)(item / ncol), tile = (int)(item - (int64_t)zcl * ncol);
-      const int64_t zc = slab_map(a, zcl);
-      const int ty = tile / a.tiles_x, tx = tile - ty * a.tiles_x;
-      const int64_t z0 = zc * C::ZCH, z1 = min(a.E0, z0 + C::ZCH);
-      for (int64_t zi = z0 - C::R; zi < z1 + C::R; ++zi) {
+    // CSX_LOCKSTEP=k (experiment): producers of all CTAs meet every k plane slots so that
+    // neighbouring tiles' halo planes are fetched while they are still in L2.  Every CTA walks the
+    // same schedule of (item round, plane slot) pairs, arriving also for the slots it has no
+    // plane for (last round, short last z chunk), so the counts match.
+    const int64_t rounds = (a.ntiles + gridDim.x - 1) / gridDim.x;
+    unsigned long long q = 0;
+    for (int64_t rr = 0; rr < rounds; ++rr) {
+      const int64_t item = blockIdx.x + rr * gridDim.x;
+      const bool has = item < a.ntiles;
+      int ty = 0, tx = 0;
+      int64_t z0 = 0, z1 = 0;
+      if (has) {
+        const int zcl = (int)(item / ncol), tile = (int)(item - (int64_t)zcl * ncol);
+        const int64_t zc = slab_map(a, zcl);
+        ty = tile / a.tiles_x;
+        tx = tile - ty * a.tiles_x;
+        z0 = zc * C::ZCH;
+        z1 = min(a.E0, z0 + C::ZCH);
+      }
+      const int64_t nsl = a.lockstep > 0 ? (int64_t)C::ZCH + 2 * C::R : (has ? z1 - z0 + 2 * C::R : 0);
+      for (int64_t p = 0; p < nsl; ++p) {
+        const int64_t zi = z0 - C::R + p;
+        const bool real = has && zi < z1 + C::R;
+        if (a.lockstep > 0 && (++q % a.lockstep) == 0) {
+          if (lane == 0) {
+            atomicAdd(g_lock_ctr, 1ull);
+            const unsigned long long target = (q / a.lockstep) * gridDim.x;
+            unsigned long long v;
+            do {
+              asm volatile("ld.acquire.gpu.global.u64 %0, [%1];\n" : "=l"(v) : "l"(g_lock_ctr) : "memory");
+            } while (v < target);
+          }
+          __syncwarp();
+        }
+        if (!real) continue;
         if (round > 0) mbar_wait(&empty[s], (uint32_t)((round - 1) & 1));
         issue_plane<C>(a, &tmap, ty, tx, zi, smem + s * C::STAGE_A, &full[s], lane);
         if (++s == C::STAGES) {
@@ -1027,6 +1058,8 @@ using Tile3D7 = Tile3DCfg<7, 4, 2, 4, 10, 32, 1, 0, 4, 2, 0>;
 // the same with the k-slice-outer DMMA order (G independent accumulator chains per k-slice)
 using Tile3D5k = Tile3DCfg<5, 4, 4, 2, 9, 32, 1, 1, 2, 4, 0>;
 using Tile3D7k = Tile3DCfg<7, 4, 2, 4, 10, 32, 1, 1, 4, 2, 0>;
+// radius 2 with twice the blocks per warp (8 accumulator chains, CTA 64 x 64, 6-plane ring)
+using Tile3D5g = Tile3DCfg<5, 8, 4, 2, 6, 32, 1, 1, 2, 4, 0>;
 
 
 // ------------------------------------------------------------------------------------------
@@ -1304,6 +1337,15 @@ static cudaError_t launch_tile3d_cfg(S2RArgs a, int tc_mask, cudaStream_t st) {
   if (a.ntiles == 0) return cudaSuccess;
   CUtensorMap tmap;
   if (!make_tmap(a, C::TP, C::RR, &tmap)) return cudaErrorNotSupported;  // 3D stages by TMA only
+  {
+    const char* ls = getenv("CSX_LOCKSTEP");
+    a.lockstep = ls ? atoi(ls) : 0;
+    if (a.lockstep > 0) {
+      void* ctr = nullptr;
+      cudaGetSymbolAddress(&ctr, g_lock_ctr);
+      cudaMemsetAsync(ctr, 0, 8, st);
+    }
+  }
   // star shapes (one TC plane) keep that plane's fragments in registers (C::WREG = 0 configs)
   auto kern = (!C::WREG && __builtin_popcount((unsigned)tc_mask) == 1) ? k_tile3d<C, true> : k_tile3d<C, false>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
@@ -1325,6 +1367,11 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
       // k-slice-outer DMMA order by default (box r = 2 / 3: 56.4 -> 60.0 / 26.6 -> 27.6 GSt/s)
       const char* e = getenv("CSX_TILE3D_KO");
       const bool ko = e ? e[0] == '1' : true;
+      // star (one TC plane): 8 blocks per warp (Star-3D13P 158 -> 180 GSt/s); box: 4 (the 9-plane
+      // ring; Box-3D125P 59.9 vs 58.4).  CSX_TILE3D5_G8 = 0 / 1 forces either.
+      const char* g8 = getenv("CSX_TILE3D5_G8");
+      const bool star = __builtin_popcount((unsigned)a.tc_mask) == 1;
+      if (nk == 5 && (g8 ? g8[0] == '1' : star)) return launch_tile3d_cfg<Tile3D5g>(a, a.tc_mask, st);
       if (nk == 5) return ko ? launch_tile3d_cfg<Tile3D5k>(a, a.tc_mask, st) : launch_tile3d_cfg<Tile3D5>(a, a.tc_mask, st);
       return ko ? launch_tile3d_cfg<Tile3D7k>(a, a.tc_mask, st) : launch_tile3d_cfg<Tile3D7>(a, a.tc_mask, st);
     }

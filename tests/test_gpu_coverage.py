@@ -167,6 +167,10 @@ def test_full_extent_parity(csx, case):
         err = rel(got, ref)
         assert err <= TOL, (name, ext, T, info["fuse_steps"], err)
         del got
+    if name == "box2d9p":  # C2 also on the paper's layout (warp-specialised TC_S2R)
+        got, info = run_gpu(csx, u0, w, s.kind, "fixed", T, engine="tc_s2r", graph=True)
+        assert info["engine_name"] == "tc_s2r"
+        assert rel(got, ref) <= TOL, (name, "tc_s2r")
 
 
 # ---- teardown: plan destruction returns every byte ------------------------------------------
