@@ -346,7 +346,7 @@ class Plan:
             raise ValueError("weights must have one axis per grid axis")
         self.radius = (w.shape[0] - 1) // 2
         self.n = int(np.prod(self.extents))
-        if fuse_steps == 0 and engine != "auto":
+        if fuse_steps == 0 and engine in ("tc_s2r", "direct"):
             # the automatic depth for the requested engine (TC_S2R 1D keeps nk + 1 <= 16)
             fuse_steps = int(_lib.csx_auto_fuse_steps(self.ndim, self.radius, ENGINES[engine]))
         self._h = csx_plan(self.ndim, self.extents, CSX_SHAPE_BOX if shape == "box" else CSX_SHAPE_STAR,

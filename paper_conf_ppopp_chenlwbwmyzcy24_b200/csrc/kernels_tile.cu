@@ -1032,6 +1032,276 @@ static cudaError_t launch_tile3d_tb(S2RArgs a, int tc_mask, cudaStream_t st) {
   return launch_pdl(a.pdl != 0, k_tile3d_tb, grid, C::NT, C::SMEM, st, a, tc_mask, tmap);
 }
 
+// ------------------------------------------------------------------------------------------
+// 3D Tf = 2 by temporal blocking, decoupled levels (round 2, k_tile3d_tb2; the default depth of
+// 3D r = 1 stars): the same two-level computation as k_tile3d_tb, but level 1 and level 2 run on
+// DIFFERENT warps that hand planes over through mbarriers instead of meeting at one CTA barrier
+// per plane, so a slow warp of one level no longer stalls the other:
+//   warp 17            producer: input planes -> IN-slot ring (TMA tensor copies)
+//   warps 8 .. 16      level 1: step-1 plane k (one row of W1 DMMA tiles of 4 x 16 per warp) from
+//                      input planes k-1 .. k+1 -> L1S-slot step-1 ring
+//   warps 0 .. 7       level 2: output plane k-1 (one row of 4 tiles per warp) from step-1 planes
+//                      k-2 .. k, stored to global memory
+// Heat-3D 512^3: 313 GSt/s (round-1 k_tile3d_tb 215, Tf = 1 k_tile3d 293).  FIXED: both levels
+// hold the frame (no band fix-up).
+template <int IN_ = 4, int L1S_ = 5, int WIDE_ = 1>
+struct Tile3DTB2 {
+  static constexpr int R = 1, A = 4, B = 2, KR = 6, KS = 6, H = 2, ZCH = 32;
+  // WIDE = 1: 32 x 64 output tile, step-1 plane 36 x 80 (level-1 warps: 5 DMMA tiles each),
+  //           inputs of output (row, col) at staged (row + dy, col + 1 + dx)   [OFF = 1]
+  // WIDE = 0: 32 x 62 output tile, step-1 plane 36 x 64 (4 tiles each: both levels equal work),
+  //           inputs at staged (row + dy, col + dx)                             [OFF = 0]
+  // (measured: WIDE = 1 312.7 GSt/s on Heat-3D, WIDE = 0 281 despite 9 % fewer DMMAs per output)
+  static constexpr int WIDE = WIDE_, OFF = WIDE_;
+  static constexpr int BM = 32, BN = WIDE_ ? 64 : 62;   // output tile (stored)
+  static constexpr int W1 = WIDE_ ? 5 : 4;               // level-1 DMMA tiles per warp
+  static constexpr int NL2 = 8, NL1 = 9;                 // level-2 / level-1 warps
+  static constexpr int NT = 32 * (NL2 + NL1 + 1);
+  static constexpr int TP = WIDE_ ? 84 : 68;             // plane pitch (input and step-1)
+  static constexpr int RIN = 38, R1 = 36;                // staged input rows, step-1 rows
+  static constexpr int SIN = RIN * TP, SIN_A = (SIN + 15) / 16 * 16;
+  static constexpr int SL1 = R1 * TP, SL1_A = (SL1 + 15) / 16 * 16;
+  // ring slots: input (3 read + IN - 3 in flight) and step-1 (3 read + 1 written + slack);
+  // measured: the step-1 slack matters, deeper input rings do not
+  static constexpr int IN = IN_, L1S = L1S_;
+  static constexpr int SMEM = (IN * SIN_A + L1S * SL1_A) * 8 + 128;
+  static_assert(SMEM <= 227 * 1024, "shared memory");
+};
+
+// G DMMA tiles of 4 x 16 outputs side by side (columns c0 + 16 j) of a plane window whose staged
+// planes pl[dz] hold the inputs of output (row, col) at (row + dy, col + OFF + dx), dy, dx in 0..2:
+// TC planes on DMMA (4x2 output blocks, K = 24), single-tap planes as DFMA on the centre cell.
+template <class C, int G, bool ONE>
+__device__ __forceinline__ void tb_hwindow(double (&acc)[G][2], const double* const (&pl)[3], int r0, int c0,
+                                           int tc_mask, const double (&wf)[ONE ? 1 : 3][6],
+                                           const double (&wz)[3], int lane) {
+  const int g = lane >> 2, t = lane & 3;
+  const int alpha = (2 * t) / C::B, beta = (2 * t) % C::B;
+#pragma unroll
+  for (int j = 0; j < G; ++j) acc[j][0] = acc[j][1] = 0.0;
+#pragma unroll
+  for (int dz = 0; dz < 3; ++dz) {
+    if (tc_mask & (1 << dz)) {
+      const double* base = pl[dz] + r0 * C::TP + c0 + C::OFF + C::B * g + t;
+#pragma unroll
+      for (int rho = 0; rho < C::KR; ++rho)
+#pragma unroll
+        for (int j = 0; j < G; ++j) dmma_t(acc[j][0], acc[j][1], base[rho * C::TP + 16 * j], wf[ONE ? 0 : dz][rho]);
+    } else if (wz[dz] != 0.0) {
+#pragma unroll
+      for (int j = 0; j < G; ++j) {
+        const double* v = pl[dz] + (r0 + alpha + C::R) * C::TP + c0 + 16 * j + C::B * g + beta + C::R + C::OFF;
+        double v0, v1;
+        if (C::OFF) {  // even centre column: one 16-B load
+          const double2 w2 = *reinterpret_cast<const double2*>(v);
+          v0 = w2.x;
+          v1 = w2.y;
+        } else {
+          v0 = v[0];
+          v1 = v[1];
+        }
+        acc[j][0] = fma(wz[dz], v0, acc[j][0]);
+        acc[j][1] = fma(wz[dz], v1, acc[j][1]);
+      }
+    }
+  }
+}
+
+template <bool ONE, class D>  // ONE: a single TC plane (star shapes): only its fragments in registers
+__global__ void __launch_bounds__(D::NT, 1)
+    k_tile3d_tb2(S2RArgs a, int tc_mask, const __grid_constant__ CUtensorMap tmap) {
+  extern __shared__ __align__(128) double smem_raw[];
+  double* smem = ring_base(smem_raw);
+  double* l1 = smem + D::IN * D::SIN_A;  // L1S step-1 planes
+  __shared__ __align__(8) uint64_t in_full[D::IN], in_empty[D::IN], l1_full[D::L1S], l1_empty[D::L1S];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  // step-1 columns 64 .. TP-1 are read (by level 2's last DMMA tile, for outputs 62, 63, which
+  // are not stored) but never written: keep them finite
+  for (int i = tid; i < D::L1S * D::R1; i += D::NT) {
+    double* row = l1 + (i / D::R1) * D::SL1_A + (i % D::R1) * D::TP;
+    for (int c = 16 * D::W1; c < D::TP; ++c) row[c] = 0.0;
+  }
+  if (tid == 0) {
+    for (int s = 0; s < D::IN; ++s) {
+      mbar_init(&in_full[s], 1);
+      mbar_init(&in_empty[s], D::NL1);
+    }
+    for (int s = 0; s < D::L1S; ++s) {
+      mbar_init(&l1_full[s], D::NL1);
+      mbar_init(&l1_empty[s], D::NL2);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  __syncthreads();
+  pdl_begin();
+  const int ncol = a.tiles_x * a.tiles_y;
+  if (warp == D::NL2 + D::NL1) {  // producer: input planes z0-2 .. z1+1 of every item
+    if (lane == 0) tma_prefetch_desc(&tmap);
+    int q = 0;
+    for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
+      const int zcl = (int)(item / ncol), tile = (int)(item - (int64_t)zcl * ncol);
+      const int64_t zc = slab_map(a, zcl);
+      const int ty = tile / a.tiles_x, tx = tile - ty * a.tiles_x;
+      const int64_t z0 = zc * D::ZCH, z1 = min(a.E0, z0 + D::ZCH);
+      for (int64_t zi = z0 - D::H; zi < z1 + D::H; ++zi, ++q) {
+        const int s = q % D::IN, n = q / D::IN;
+        if (n > 0) mbar_wait(&in_empty[s], (uint32_t)((n - 1) & 1));
+        if (lane == 0) {
+          mbar_expect_tx(&in_full[s], (uint32_t)(D::SIN * 8));
+          tma_load_3d(smem + s * D::SIN_A, &tmap, &in_full[s], (int)(a.tma_x0 + (int64_t)tx * D::BN - 2 - 2 * D::OFF),
+                      (int)(a.tma_y0 + (int64_t)ty * D::BM - 2), (int)(a.tma_z0 + zi));
+        }
+      }
+    }
+    return;
+  }
+  double wf[ONE ? 1 : 3][D::KS], wz[3];
+  const int dz1 = __ffs(tc_mask) - 1;
+#pragma unroll
+  for (int p = 0; p < (ONE ? 1 : 3); ++p)
+#pragma unroll
+    for (int k = 0; k < D::KS; ++k) wf[p][k] = a.frags[((ONE ? dz1 : p) * D::KS + k) * 32 + lane];
+#pragma unroll
+  for (int p = 0; p < 3; ++p) wz[p] = a.wc[(p * 3 + 1) * 3 + 1];
+  const int g = lane >> 2, t = lane & 3;
+  const int alpha = (2 * t) / D::B, beta = (2 * t) % D::B;
+  const bool fixed = a.hold_frame != 0;
+  if (warp >= D::NL2) {
+    // ---------------- level 1: step-1 planes ----------------
+    const int rb = warp - D::NL2;  // step-1 rows 4 rb .. 4 rb + 3, cols 0 .. 16 W1 - 1
+    int q = 0, p = 0;              // input / step-1 plane sequence numbers
+    for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
+      const int zcl = (int)(item / ncol), tile = (int)(item - (int64_t)zcl * ncol);
+      const int64_t zc = slab_map(a, zcl);
+      const int ty = tile / a.tiles_x, tx = tile - ty * a.tiles_x;
+      const int64_t z0 = zc * D::ZCH, z1 = min(a.E0, z0 + D::ZCH);
+      // global origin of the step-1 plane: (y0 - 1, x0 - 1 - OFF)
+      const int64_t sy0 = (int64_t)ty * D::BM + a.gorg1 - 1, sx0 = (int64_t)tx * D::BN + a.gorg2 - 1 - D::OFF;
+      const bool tile_edge =
+          fixed && (sy0 < 1 || sy0 + D::R1 > a.GE1 - 1 || sx0 < 1 || sx0 + 16 * D::W1 > a.GE2 - 1);
+      const int q0 = q;  // input plane z0-2 of this item
+      auto in_slot = [&](int qq) { return smem + (qq % D::IN) * D::SIN_A; };
+      mbar_wait(&in_full[q0 % D::IN], (uint32_t)((q0 / D::IN) & 1));
+      mbar_wait(&in_full[(q0 + 1) % D::IN], (uint32_t)(((q0 + 1) / D::IN) & 1));
+      // step-1 plane k (k = z0-1 .. z1) from input planes k-1, k, k+1 (sequence q0 + j, +1, +2)
+      for (int64_t k = z0 - 1; k <= z1; ++k, ++p) {
+        const int j = (int)(k - (z0 - 1));
+        mbar_wait(&in_full[(q0 + j + 2) % D::IN], (uint32_t)(((q0 + j + 2) / D::IN) & 1));
+        const int sl = p % D::L1S, nl = p / D::L1S;
+        if (nl > 0) mbar_wait(&l1_empty[sl], (uint32_t)((nl - 1) & 1));
+        const double* pin[3] = {in_slot(q0 + j), in_slot(q0 + j + 1), in_slot(q0 + j + 2)};
+        double* dl1 = l1 + sl * D::SL1_A;
+        double acc[D::W1][2];
+        tb_hwindow<D, D::W1, ONE>(acc, pin, 4 * rb, 0, tc_mask, wf, wz, lane);
+        const int64_t gz1 = k + a.gorg0;
+        const bool zf1 = fixed && (gz1 < 1 || gz1 >= a.GE0 - 1);
+#pragma unroll
+        for (int jj = 0; jj < D::W1; ++jj) {
+          const int r = 4 * rb + alpha, c = 16 * jj + D::B * g + beta;  // step-1 plane coords
+          double v0 = acc[jj][0], v1 = acc[jj][1];
+          if (fixed && (zf1 || tile_edge)) {  // held frame points keep the input value
+            const int64_t gy = sy0 + r, gx = sx0 + c;
+            const double* ctr = pin[1] + (r + 1) * D::TP + c + 1 + D::OFF;
+            const bool yf = zf1 || gy < 1 || gy >= a.GE1 - 1;
+            if (yf || gx < 1 || gx >= a.GE2 - 1) v0 = ctr[0];
+            if (yf || gx + 1 < 1 || gx + 1 >= a.GE2 - 1) v1 = ctr[1];
+          }
+          *reinterpret_cast<double2*>(dl1 + r * D::TP + c) = make_double2(v0, v1);
+        }
+        __syncwarp();
+        if (lane == 0) {
+          mbar_arrive(&l1_full[sl]);                    // this warp's rows of plane k written
+          mbar_arrive(&in_empty[(q0 + j) % D::IN]);     // input plane k-1 no longer read
+        }
+      }
+      __syncwarp();
+      if (lane == 0) {  // input planes z1, z1+1 (read by the last step-1 plane only)
+        mbar_arrive(&in_empty[(q0 + (int)(z1 - z0) + 2) % D::IN]);
+        mbar_arrive(&in_empty[(q0 + (int)(z1 - z0) + 3) % D::IN]);
+      }
+      q = q0 + (int)(z1 - z0) + 4;
+    }
+    return;
+  }
+  // ---------------- level 2: output planes ----------------
+  const int rb = warp;  // output rows 4 rb .. 4 rb + 3, cols 0 .. 63 (BN stored)
+  int p = 0;            // step-1 plane sequence number
+  for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
+    const int zcl = (int)(item / ncol), tile = (int)(item - (int64_t)zcl * ncol);
+    const int64_t zc = slab_map(a, zcl);
+    const int ty = tile / a.tiles_x, tx = tile - ty * a.tiles_x;
+    const int64_t z0 = zc * D::ZCH, z1 = min(a.E0, z0 + D::ZCH);
+    const int64_t y0 = (int64_t)ty * D::BM, x0 = (int64_t)tx * D::BN;
+    const int64_t gy0 = y0 + a.gorg1, gx0 = x0 + a.gorg2;
+    const bool tile_edge = fixed && (gy0 < 1 || gy0 + D::BM > a.GE1 - 1 || gx0 < 1 || gx0 + D::BN > a.GE2 - 1);
+    const int p0 = p;  // step-1 plane z0-1 of this item
+    auto l1_slot = [&](int pp) { return l1 + (pp % D::L1S) * D::SL1_A; };
+    auto l1_wait = [&](int pp) { mbar_wait(&l1_full[pp % D::L1S], (uint32_t)((pp / D::L1S) & 1)); };
+    l1_wait(p0);
+    l1_wait(p0 + 1);
+    for (int64_t zo = z0; zo < z1; ++zo) {
+      const int j = (int)(zo - z0);
+      l1_wait(p0 + j + 2);
+      const double* p1[3] = {l1_slot(p0 + j), l1_slot(p0 + j + 1), l1_slot(p0 + j + 2)};
+      double acc[4][2];
+      tb_hwindow<D, 4, ONE>(acc, p1, 4 * rb, 0, tc_mask, wf, wz, lane);
+      const int64_t gzo = zo + a.gorg0;
+      const bool zf = fixed && (gzo < 1 || gzo >= a.GE0 - 1);
+      double* plane = a.dst.p + zo * a.dst.s0;
+#pragma unroll
+      for (int jj = 0; jj < 4; ++jj) {
+        const int r = 4 * rb + alpha, c = 16 * jj + D::B * g + beta;  // output tile coords
+        if (c >= D::BN) continue;  // columns 62, 63 are the neighbour tile's
+        const int64_t row = y0 + r, col = x0 + c;
+        double v0 = acc[jj][0], v1 = acc[jj][1];
+        if (fixed && (zf || tile_edge)) {
+          const double* ctr = p1[1] + (r + 1) * D::TP + c + 1 + D::OFF;
+          const int64_t gy = gy0 + r, gx = gx0 + c;
+          const bool yf = zf || gy < 1 || gy >= a.GE1 - 1;
+          if (yf || gx < 1 || gx >= a.GE2 - 1) v0 = ctr[0];
+          if (yf || gx + 1 < 1 || gx + 1 >= a.GE2 - 1) v1 = ctr[1];
+        }
+        if (row >= a.E1 || col >= a.E2) continue;
+        double* pp = plane + row * a.dst.s1 + col;
+        if (col + 1 < a.E2 && a.dst_aligned) {
+          *reinterpret_cast<double2*>(pp) = make_double2(v0, v1);
+        } else {
+          pp[0] = v0;
+          if (col + 1 < a.E2) pp[1] = v1;
+        }
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&l1_empty[(p0 + j) % D::L1S]);  // step-1 plane zo-1 done
+    }
+    __syncwarp();
+    if (lane == 0) {  // step-1 planes z1-1, z1 (read by the last output plane only)
+      mbar_arrive(&l1_empty[(p0 + (int)(z1 - z0)) % D::L1S]);
+      mbar_arrive(&l1_empty[(p0 + (int)(z1 - z0) + 1) % D::L1S]);
+    }
+    p = p0 + (int)(z1 - z0) + 2;
+  }
+}
+
+template <class D>
+static cudaError_t launch_tile3d_tb2(S2RArgs a, int tc_mask, cudaStream_t st) {
+  a.dst_aligned = ((reinterpret_cast<uintptr_t>(a.dst.p) & 15) == 0) && (a.dst.s1 % 2 == 0) &&
+                  (a.dst.s0 % 2 == 0);
+  a.tiles_x = (int)((a.E2 + D::BN - 1) / D::BN);
+  a.tiles_y = (int)((a.E1 + D::BM - 1) / D::BM);
+  a.ntiles = (int64_t)a.tiles_x * a.tiles_y * set_ranges(a, (a.E0 + D::ZCH - 1) / D::ZCH, D::ZCH, a.E0, D::H);
+  if (a.ntiles == 0) return cudaSuccess;
+  CUtensorMap tmap;
+  if (!make_tmap(a, D::TP, D::RIN, &tmap)) return cudaErrorNotSupported;
+  auto kern = __builtin_popcount((unsigned)tc_mask) == 1 ? k_tile3d_tb2<true, D> : k_tile3d_tb2<false, D>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, D::SMEM);
+  if (e != cudaSuccess) return e;
+  int occ = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, D::NT, D::SMEM);
+  if (e != cudaSuccess) return e;
+  const int64_t grid = persistent_grid(occ, a.max_ctas, a.ntiles);
+  return launch_pdl(a.pdl != 0, kern, grid, D::NT, D::SMEM, st, a, tc_mask, tmap);
+}
+
 using Tile3D3 = Tile3DCfg<3, 8, 2, 2, 5, 32>;      // CTA 64 x 32 outputs, 4 DMMA warps, 5-plane ring, 32 planes per item
 using Tile3D3b = Tile3DCfg<3, 4, 4, 1, 5, 32, 2>;  // CTA 64 x 32, 4 warps of 4 block rows x 2 column groups
 using Tile3D3c = Tile3DCfg<3, 8, 2, 4, 6, 32>;     // CTA 64 x 64 outputs, 8 DMMA warps, 6-plane ring
@@ -1362,7 +1632,13 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
   const int nk = 2 * radius * tf + 1;
   if (ndim == 1) return launch_tile1d(nk, a, st);
   if (ndim == 3) {
-    if (tf == 2) return launch_tile3d_tb<Tile3DTB>(a, a.tc_mask, st);  // r = 1: temporal blocking
+    if (tf == 2) {  // r = 1: temporal blocking (CSX_TB=1: the round-1 single-barrier kernel)
+      const char* e = getenv("CSX_TB");
+      if (e && e[0] == '1') return launch_tile3d_tb<Tile3DTB>(a, a.tc_mask, st);
+      const char* r = getenv("CSX_TB_GEOM");  // 0: the 32 x 62 tile (equal level work)
+      if (r && r[0] == '0') return launch_tile3d_tb2<Tile3DTB2<5, 6, 0>>(a, a.tc_mask, st);
+      return launch_tile3d_tb2<Tile3DTB2<4, 5, 1>>(a, a.tc_mask, st);
+    }
     if (nk == 5 || nk == 7) {
       // k-slice-outer DMMA order by default (box r = 2 / 3: 56.4 -> 60.0 / 26.6 -> 27.6 GSt/s)
       const char* e = getenv("CSX_TILE3D_KO");

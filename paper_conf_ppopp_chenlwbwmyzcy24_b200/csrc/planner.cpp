@@ -344,7 +344,20 @@ int auto_tf(int ndim, int radius, int engine) {
 }
 
 csx_status build_plan(csx_plan_s* p) {
-  if (p->tf <= 0) p->tf = auto_tf(p->ndim, p->radius, CSX_ENGINE_AUTO);
+  if (p->tf <= 0) {
+    p->tf = auto_tf(p->ndim, p->radius, CSX_ENGINE_AUTO);
+    // 3D r = 1 stars (single-tap z arms: one TC plane): two steps per pass by temporal blocking
+    // (k_tile3d_tb2, Heat-3D 313 vs 293 GSt/s at Tf = 1); boxes keep Tf = 1 (150 vs 196)
+    if (p->ndim == 3 && p->radius == 1) {
+      bool star = true;
+      for (int dz = 0; dz < 3; dz += 2) {
+        int taps = 0;
+        for (int i = 0; i < 9; ++i) taps += p->w[(size_t)dz * 9 + i] != 0.0;
+        star = star && taps <= 1;
+      }
+      if (star) p->tf = 2;
+    }
+  }
   const int nk = 2 * p->radius * p->tf + 1;
   // 1D: TC_S2R (the paper's layout, nf <= 2 N fragments) takes nk <= 15, TC_TILE (Toeplitz
   // blocks) nk <= 31 — the FIXED band code's 32-lane cone needs 2 r (Tf-1) <= 31.

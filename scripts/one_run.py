@@ -20,12 +20,13 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", required=True)
 ap.add_argument("--engine", default="auto")
 ap.add_argument("--T", type=int, default=None)
+ap.add_argument("--fuse", type=int, default=None)
 args = ap.parse_args()
 shape, ext, T, bc, tf = bench.CONFIGS[args.config]
 T = args.T or T
 s = synth.SHAPES[shape]
 w = synth.physical_weights(shape)
-p = csx.Plan(ext, w, shape=s.kind, bc=bc, fuse_steps=tf, engine=args.engine)
+p = csx.Plan(ext, w, shape=s.kind, bc=bc, fuse_steps=tf if args.fuse is None else args.fuse, engine=args.engine)
 d_in = synth.grid_torch(ext, "cuda")
 d_out = torch.empty_like(d_in)
 p.run(d_in, d_out, T)

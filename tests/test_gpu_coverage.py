@@ -236,3 +236,18 @@ def test_graph_plan_variant_switch_teardown(csx):
     # 8 cycles: any leaked grid (>= 2.8 MB) or stencil2row scratch (~5 MB) adds up past 8 MB
     leak = base - _free_bytes()
     assert leak < (8 << 20), f"{leak >> 20} MB not returned"
+
+
+@pytest.mark.parametrize("env", [{"CSX_TILE3D_KO": "0"}, {"CSX_TILE3D5_G8": "1"}, {"CSX_TILE3D5_G8": "0"}])
+def test_parity_3d_general_radius_variants(csx, monkeypatch, env):
+    """The other 3D r = 2 / 3 tile configurations (row-outer DMMA order; 8 or 4 blocks per warp
+    for both stars and boxes; read at every launch): ragged tiles and z chunks, both boundaries."""
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    for name in R3D:
+        s = synth.SHAPES[name]
+        w = synth.random_weights(name)
+        u0 = synth.grid((40, 70, 90), seed=601)
+        for bc in ("fixed", "periodic"):
+            got, _ = run_gpu(csx, u0, w, s.kind, bc, 2, engine="tc_tile", max_ctas=5)
+            assert rel(got, oracle.run(u0, w, bc, 2)) <= TOL, (name, bc, env)

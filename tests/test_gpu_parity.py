@@ -296,7 +296,7 @@ def test_parity_3d_tile_variants(csx, monkeypatch, variant):
         u0 = synth.grid(ext, seed=33)
         w = synth.random_weights(name)
         for bc in ("fixed", "periodic"):
-            got, info = run_gpu(csx, u0, w, s.kind, bc, 3, engine="tc_tile")
+            got, info = run_gpu(csx, u0, w, s.kind, bc, 3, engine="tc_tile", fuse_steps=1)
             assert rel(got, oracle.run(u0, w, bc, 3)) <= TOL, (name, ext, bc, variant)
 
 
@@ -308,7 +308,7 @@ def test_parity_3d_zchunks(csx, name, engine):
     u0 = synth.grid((70, 37, 45), seed=31)
     w = synth.random_weights(name)
     for bc in ("fixed", "periodic"):
-        got, info = run_gpu(csx, u0, w, s.kind, bc, 4, engine=engine)
+        got, info = run_gpu(csx, u0, w, s.kind, bc, 4, engine=engine, fuse_steps=1)
         assert info["engine_name"] == engine
         assert rel(got, oracle.run(u0, w, bc, 4)) <= TOL, (name, engine, bc)
 

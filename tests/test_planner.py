@@ -257,8 +257,9 @@ def test_2d_fusion_limits():
 
 
 def test_auto_fusion_depths():
+    # (3D r = 1 stars run two steps per pass by temporal blocking; boxes and r >= 2 one)
     cases = {"heat1d": 11, "1d5p": 5, "heat2d": 3, "box2d9p": 3, "star2d13p": 1, "box2d49p": 1,
-             "heat3d": 1, "box3d27p": 1}
+             "heat3d": 2, "box3d27p": 1, "star3d13p": 1, "box3d125p": 1}
     for name, tf in cases.items():
         s = synth.SHAPES[name]
         ext = {1: (4096,), 2: (128, 128), 3: (32, 32, 32)}[s.ndim]
@@ -271,6 +272,11 @@ def test_auto_fusion_depths():
         assert p.info()["fuse_steps"] == tf and p.info()["engine_name"] == "tc_s2r", name
         p.close()
     assert csx._lib.csx_auto_fuse_steps(1, 3, csx.ENGINES["tc_tile"]) == 3
+    # the CUDA-core comparator's own depth (2D r = 1: 4 steps)
+    assert csx._lib.csx_auto_fuse_steps(2, 1, csx.ENGINES["direct"]) == 4
+    p = csx.Plan((64, 64), synth.physical_weights("box2d9p"), engine="direct")
+    assert p.info()["fuse_steps"] == 4
+    p.close()
     assert csx._lib.csx_auto_fuse_steps(4, 1, 0) == 0
 
 
