@@ -381,7 +381,8 @@ def main():
         lo, hi = plan.shard_box(rank, p0, p1)
         u0 = np.ascontiguousarray(synth.grid(gext, rows=(lo[0], hi[0]))[:, lo[1]:hi[1]])
     elif world > 1:
-        exchange = "peer" if args.exchange == "peer" else "nccl"
+        # shared-GPU test mode (ranks on one GPU): NCCL cannot put two ranks on one device
+        exchange = "peer" if (args.exchange == "peer" or share) else "nccl"
         if exchange == "peer":
             # halo exchange by SM peer stores over NVLink (CUDA IPC), epoch flags in peer memory;
             # if the IPC mapping is refused, every rank switches to the NCCL exchange
@@ -498,9 +499,9 @@ def main():
             # graph replay carries no per-kernel events: the dominant kernel's share of the extra
             # eager step, applied to the replayed step's time (an eager step is slower than its
             # replay when it is launch-bound, e.g. the 1D configs' short passes)
-            share = min(1.0, tc_ms / eager_ms)
+            kshare = min(1.0, tc_ms / eager_ms)
             avg_eager_ms = tc_ms / tc_launches
-            avg_s = share * ms_step / tc_launches * 1e-3
+            avg_s = kshare * ms_step / tc_launches * 1e-3
         mma = algorithmic_mma(s.ndim, nk, tfm, engine, local_points, tcp)
         mma_src = ("Eq 13 generalised (reading A7, 3D planes)" if engine == "tc_s2r" else
                    "TC_TILE block count: K of the a x b output block / 4 per 64 outputs")
@@ -531,7 +532,7 @@ def main():
                     "per_launch": f"16 B x {local_points} points (1 read + 1 write per pass)",
                     "tensor_frac": flops / avg_s / 1e12 / dmma}
         if eager_ms:
-            roof["tc_share_of_step"] = share
+            roof["tc_share_of_step"] = kshare
             roof["timing"] = ("dominant-kernel share of one eager profiled step x the replayed "
                               "step time / launches per step")
             roof["avg_launch_ms_eager"] = avg_eager_ms
@@ -698,7 +699,7 @@ def main():
                            "h2d_bytes_per_step": int(u0.nbytes), "d2h_bytes_per_step": int(u0.nbytes),
                            "api": "torch pinned copies + csx_run_sharded" + ("_peer" if comm is None else ""),
                            "ms_per_step": ems}
-    if world > 1 and not pencil and args.exchange == "both":
+    if world > 1 and not pencil and args.exchange == "both" and not share:
         # the same weak-scaled step with the halo exchange fused into SM peer stores over NVLink
         # (csx_run_sharded_peer), timed the same way (max over ranks); the line's value is the
         # NCCL run above (the north_star path)

@@ -401,6 +401,140 @@ __global__ void __launch_bounds__(128, 4) k_s2r1d(S2RArgs a) {
 }
 
 // ------------------------------------------------------------------------------------------
+// 1D, warp-specialised (default): the tile's input run (contiguous in 1D) arrives by ONE bulk
+// copy into a 2-stage raw ring, dedicated scatter warps run the LUT scatter smem -> smem into
+// one of two A/B buffers while the DMMA warps tessellate the other (round 1 gathered every LUT
+// element with its own __ldg from global memory, synchronously, between two CTA barriers).
+template <int NK>
+struct S2R1DWS {
+  using G = S2R1D<NK>;
+  static constexpr int ODD = G::R & 1;                       // 16-B aligned copy start
+  static constexpr int RAWN = (ODD + G::RC + 1) / 2 * 2;     // staged doubles (16-B multiple)
+  static constexpr int RAW_A = (RAWN + 15) / 16 * 16;        // 128-B aligned ring slots
+  static constexpr int NCW = 8, NSW = 2;                     // DMMA warps, scatter warps
+  static constexpr int NT = 32 * (NCW + NSW + 1);
+  static constexpr int AB = 2 * (G::STRIPS + 1) * G::PITCH;  // doubles per A/B buffer
+  static constexpr int SMEM = 2 * RAW_A * 8 + 2 * AB * 8 + G::NE * 4 + 128;
+};
+
+template <int NK>
+__global__ void __launch_bounds__(S2R1DWS<NK>::NT, 1) k_s2r1d_ws(S2RArgs a) {
+  using G = S2R1D<NK>;
+  using W = S2R1DWS<NK>;
+  constexpr int NF = G::NF, KS = G::KS;
+  extern __shared__ __align__(128) double smem_raw1[];
+  double* raw = smem_raw1 + ((128u - (s2r_smem_u32(smem_raw1) & 127u)) & 127u) / 8u;  // 2 x RAW_A
+  double* sAB = raw + 2 * W::RAW_A;                                                   // 2 x AB
+  uint32_t* sL = reinterpret_cast<uint32_t*>(sAB + 2 * W::AB);
+  __shared__ __align__(8) uint64_t full[2], empty[2], ab_full[2], ab_empty[2];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  for (int i = tid; i < 2 * W::AB; i += W::NT) sAB[i] = 0.0;
+  for (int i = tid; i < G::NE; i += W::NT) sL[i] = (uint32_t)a.lut[i].y;
+  if (tid == 0) {
+    for (int s = 0; s < 2; ++s) {
+      s2r_mbar_init(&full[s], 1);
+      s2r_mbar_init(&empty[s], W::NSW);
+      s2r_mbar_init(&ab_full[s], W::NSW);
+      s2r_mbar_init(&ab_empty[s], W::NCW);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  __syncthreads();
+  if (warp == W::NCW + W::NSW) {  // producer: one bulk copy per tile
+    int it = 0;
+    for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
+      const int s = it & 1, n = it >> 1;
+      if (n > 0) s2r_mbar_wait(&empty[s], (n - 1) & 1);
+      if (lane == 0) {
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(s2r_smem_u32(&full[s])),
+                     "r"((uint32_t)(W::RAWN * 8))
+                     : "memory");
+        asm volatile(
+            "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n" ::"r"(
+                s2r_smem_u32(raw + s * W::RAW_A)),
+            "l"(a.src.p + tile * G::BN - G::R - W::ODD), "r"((uint32_t)(W::RAWN * 8)), "r"(s2r_smem_u32(&full[s]))
+            : "memory");
+      }
+    }
+    return;
+  }
+  if (warp >= W::NCW) {  // scatter warps: implicit stencil2row through the LUT (branch-free)
+    const int sw = warp - W::NCW;
+    int it = 0;
+    for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
+      const int s = it & 1, b = it & 1;
+      if (it >= 2) s2r_mbar_wait(&ab_empty[b], ((it >> 1) - 1) & 1);
+      s2r_mbar_wait(&full[s], (it >> 1) & 1);
+      double* sA = sAB + b * W::AB;
+      double* sB = sA + (G::STRIPS + 1) * G::PITCH;
+      const double* rs = raw + s * W::RAW_A + W::ODD;
+#pragma unroll 4
+      for (int e = sw * 32 + lane; e < G::NE; e += 32 * W::NSW) {
+        const double v = rs[e];
+        const uint32_t l = sL[e];
+        sA[l & 0xffffu] = v;
+        sB[l >> 16] = v;
+      }
+      __syncwarp();
+      if (lane == 0) {
+        s2r_mbar_arrive(&empty[s]);
+        s2r_mbar_arrive(&ab_full[b]);
+      }
+    }
+    return;
+  }
+  double wa[NF][KS], wb[NF][KS];
+#pragma unroll
+  for (int f = 0; f < NF; ++f)
+#pragma unroll
+    for (int s = 0; s < KS; ++s) {
+      wa[f][s] = a.frags[((0 * NF + f) * KS + s) * 32 + lane];
+      wb[f][s] = a.frags[((1 * NF + f) * KS + s) * 32 + lane];
+    }
+  const int g = lane >> 2, t = lane & 3;
+  int it = 0;
+  for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
+    const int b = it & 1;
+    s2r_mbar_wait(&ab_full[b], (it >> 1) & 1);
+    const double* sA = sAB + b * W::AB;
+    const double* sB = sA + (G::STRIPS + 1) * G::PITCH;
+    double c[G::NDT / W::NCW][NF][2];
+#pragma unroll
+    for (int u = 0; u < G::NDT / W::NCW; ++u) {
+      const int d = warp + u * W::NCW;
+      const double* pa = sA + (8 * d + g) * G::PITCH + t;
+      const double* pb = sB + (8 * d + g) * G::PITCH + t;
+#pragma unroll
+      for (int f = 0; f < NF; ++f) c[u][f][0] = c[u][f][1] = 0.0;
+#pragma unroll
+      for (int s = 0; s < KS; ++s) {
+        const double x = pa[4 * s];
+#pragma unroll
+        for (int f = 0; f < NF; ++f) dmma(c[u][f][0], c[u][f][1], x, wa[f][s]);
+      }
+#pragma unroll
+      for (int s = 0; s < KS; ++s) {
+        const double x = pb[4 * s];
+#pragma unroll
+        for (int f = 0; f < NF; ++f) dmma(c[u][f][0], c[u][f][1], x, wb[f][s]);
+      }
+    }
+    __syncwarp();
+    if (lane == 0) s2r_mbar_arrive(&ab_empty[b]);
+#pragma unroll
+    for (int u = 0; u < G::NDT / W::NCW; ++u) {
+      const int d = warp + u * W::NCW;
+      const int64_t o = tile * G::BN + (int64_t)(8 * d + g) * G::SW;
+#pragma unroll
+      for (int f = 0; f < NF; ++f) {
+        const int cc = 8 * f + 2 * t;
+        store_pair(a.dst.p, o + cc, a.E2, cc < G::SW, cc + 1 < G::SW, c[u][f][0], c[u][f][1]);
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------
 // 3D (Tf = 1): stream input planes along z; input plane zi contributes to output planes
 // zo = zi - R + j with the 2D weights of z offset dz = NK-1-j (P.1788-1800).  Accumulators of
 // the NK live output planes rotate in registers.  Planes whose weights are a single centre tap
@@ -596,6 +730,17 @@ cudaError_t launch_s2r(int ndim, int nk, int nf, const S2RArgs& a, int tc_mask, 
   (void)nf;
   const int smem = s2r_smem_bytes(ndim, nk, nf);
   if (smem < 0) return cudaErrorInvalidValue;
+  if (ndim == 1 && s2r_ws()) {
+    switch (nk) {
+      case 3: return launch_persistent(k_s2r1d_ws<3>, S2R1DWS<3>::SMEM, S2R1DWS<3>::NT, a.ntiles, st, a);
+      case 5: return launch_persistent(k_s2r1d_ws<5>, S2R1DWS<5>::SMEM, S2R1DWS<5>::NT, a.ntiles, st, a);
+      case 7: return launch_persistent(k_s2r1d_ws<7>, S2R1DWS<7>::SMEM, S2R1DWS<7>::NT, a.ntiles, st, a);
+      case 9: return launch_persistent(k_s2r1d_ws<9>, S2R1DWS<9>::SMEM, S2R1DWS<9>::NT, a.ntiles, st, a);
+      case 11: return launch_persistent(k_s2r1d_ws<11>, S2R1DWS<11>::SMEM, S2R1DWS<11>::NT, a.ntiles, st, a);
+      case 13: return launch_persistent(k_s2r1d_ws<13>, S2R1DWS<13>::SMEM, S2R1DWS<13>::NT, a.ntiles, st, a);
+      case 15: return launch_persistent(k_s2r1d_ws<15>, S2R1DWS<15>::SMEM, S2R1DWS<15>::NT, a.ntiles, st, a);
+    }
+  }
   if (ndim == 1) {
     switch (nk) {
       case 3: return launch_persistent(k_s2r1d<3>, smem, 128, a.ntiles, st, a);

@@ -309,17 +309,17 @@ csx_status build_pass(const csx_plan_s* p, int tf, Pass* out) {
     P.tile_mma_per_pass = (int64_t)((double)pts / 64.0 * P.tile_ks * tcp + 0.5);
   }
   if (ndim == 3 && tf == 2 && p->radius == 1) {
-    // 3D Tf = 2 runs the BASE stencil twice by temporal blocking (k_tile3d_tb), not the composed
-    // window: per 32 x 64 output tile and plane, level 1 computes 15 units x 3 blocks on the
-    // grown 36 x 80 tile and level 2 8 warps x 4 blocks, 6 DMMAs (K = 24) per block and TC plane
-    // of the base window.
+    // 3D Tf = 2 runs the BASE stencil twice by temporal blocking (k_tile3d_tb2), not the composed
+    // window: per 32 x 64 output tile and plane, level 1 computes 45 DMMA tiles (4 x 16) on the
+    // grown 36 x 80 tile for 34 of every 32 planes (the z-chunk's two extra step-1 planes) and
+    // level 2 32 tiles, 6 DMMAs (K = 24) per tile and TC plane of the base window.
     int base_tc = 0;
     for (int dz = 0; dz < 3; ++dz) {
       int taps = 0;
       for (int i = 0; i < 9; ++i) taps += p->w[(size_t)dz * 9 + i] != 0.0;
       base_tc += taps > 1;
     }
-    P.tile_mma_per_pass = (int64_t)((double)pts / 2048.0 * (15 * 3 + 8 * 4) * 6 * base_tc + 0.5);
+    P.tile_mma_per_pass = (int64_t)((double)pts / 2048.0 * (45.0 * 34.0 / 32.0 + 32.0) * 6 * base_tc + 0.5);
   }
   *out = std::move(P);
   return CSX_OK;
