@@ -639,6 +639,149 @@ __global__ void __launch_bounds__(128, 3) k_s2r3d(S2RArgs a, int tc_mask) {
 }
 
 // ------------------------------------------------------------------------------------------
+// 3D with a staged plane ring (default; CSX_S2R_WS=0 = the kernel above): a producer warp
+// streams each input plane's raw region (RR rows, one cp.async.bulk per row) into a STAGES-deep
+// ring, so the plane loads are in flight while earlier planes are scattered and tessellated
+// (k_s2r3d gathers every LUT element from global memory between two CTA barriers, exposing the
+// load latency once per plane).  The 4 compute warps scatter plane k through the LUT into A/B
+// buffer k & 1 (smem -> smem), meet at one named barrier, and run the dual tessellations of the
+// NK accumulating output planes; the single-tap planes read the staged raw region directly.
+template <int NK>
+struct S2R3DWS {
+  using G = S2R3D<NK>;
+  static constexpr int ODD = G::R & 1;
+  static constexpr int TP = (ODD + G::RC + 1) / 2 * 2;   // staged row length (16-B multiple)
+  static constexpr int RAW = G::RR * TP;
+  static constexpr int RAW_A = (RAW + 15) / 16 * 16;
+  static constexpr int STAGES = 4;
+  static constexpr int NCW = 4;
+  static constexpr int NT = 32 * (NCW + 1);
+  static constexpr int AB = 2 * (G::STRIPS + 1) * G::PITCH;
+  static constexpr int SMEM = STAGES * RAW_A * 8 + 2 * AB * 8 + G::NE * 4 + 128;
+};
+
+template <int NK>
+__global__ void __launch_bounds__(S2R3DWS<NK>::NT, 3) k_s2r3d_ws(S2RArgs a, int tc_mask) {
+  using G = S2R3D<NK>;
+  using W = S2R3DWS<NK>;
+  constexpr int KS = G::KS, R = G::R;
+  extern __shared__ __align__(128) double smem_raw3[];
+  double* raw = smem_raw3 + ((128u - (s2r_smem_u32(smem_raw3) & 127u)) & 127u) / 8u;  // STAGES x RAW_A
+  double* sAB = raw + W::STAGES * W::RAW_A;                                            // 2 x AB
+  uint32_t* sL = reinterpret_cast<uint32_t*>(sAB + 2 * W::AB);
+  __shared__ __align__(8) uint64_t full[W::STAGES], empty[W::STAGES];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  for (int i = tid; i < 2 * W::AB; i += W::NT) sAB[i] = 0.0;
+  for (int i = tid; i < G::NE; i += W::NT) sL[i] = (uint32_t)a.lut[i].y;
+  if (tid == 0) {
+    for (int s = 0; s < W::STAGES; ++s) {
+      s2r_mbar_init(&full[s], 1);
+      s2r_mbar_init(&empty[s], W::NCW);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  __syncthreads();
+  const int64_t ncol = (int64_t)a.tiles_x * a.tiles_y;
+  if (warp == W::NCW) {  // producer: raw regions of planes z0-R .. z1+R-1 of every item
+    int q = 0;
+    for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
+      const int64_t zc = item / ncol, tile = item - zc * ncol;
+      const int ty = (int)(tile / a.tiles_x), tx = (int)(tile - (int64_t)ty * a.tiles_x);
+      const int64_t z0 = zc * G::ZCHUNK, z1 = min(a.E0, z0 + G::ZCHUNK);
+      const double* base2 = a.src.p + (int64_t)(ty * G::BM - R) * a.src.s1 + (tx * G::BN - R - W::ODD);
+      for (int64_t zi = z0 - R; zi < z1 + R; ++zi, ++q) {
+        const int s = q % W::STAGES, n = q / W::STAGES;
+        if (n > 0) s2r_mbar_wait(&empty[s], (n - 1) & 1);
+        s2r_issue_rows(base2 + zi * a.src.s0, a.src.s1, raw + s * W::RAW_A, G::RR, W::TP, &full[s], lane);
+      }
+    }
+    return;
+  }
+  double wa[NK][KS], wb[NK][KS], wz[NK];
+#pragma unroll
+  for (int p = 0; p < NK; ++p) {
+#pragma unroll
+    for (int s = 0; s < KS; ++s) {
+      wa[p][s] = a.frags[((p * 2 + 0) * KS + s) * 32 + lane];
+      wb[p][s] = a.frags[((p * 2 + 1) * KS + s) * 32 + lane];
+    }
+    wz[p] = a.wc[(p * NK + R) * NK + R];
+  }
+  const int g = lane >> 2, t = lane & 3;
+  const bool v0 = 2 * t < G::SW, v1 = 2 * t + 1 < G::SW;
+  int q = 0;  // input plane sequence number (producer order)
+  for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
+    const int64_t zc = item / ncol, tile = item - zc * ncol;
+    const int ty = (int)(tile / a.tiles_x), tx = (int)(tile - (int64_t)ty * a.tiles_x);
+    const int64_t z0 = zc * G::ZCHUNK, z1 = min(a.E0, z0 + G::ZCHUNK);
+    double acc[NK][2][2];
+#pragma unroll
+    for (int j = 0; j < NK; ++j) acc[j][0][0] = acc[j][0][1] = acc[j][1][0] = acc[j][1][1] = 0.0;
+    const int xr = warp * 2;
+    const int64_t col = (int64_t)tx * G::BN + g * G::SW + 2 * t;
+    for (int64_t zi = z0 - R; zi < z1 + R; ++zi, ++q) {
+      const int s = q % W::STAGES;
+      s2r_mbar_wait(&full[s], (q / W::STAGES) & 1);
+      const double* rs = raw + s * W::RAW_A + W::ODD;
+      double* sA = sAB + (q & 1) * W::AB;
+      double* sB = sA + (G::STRIPS + 1) * G::PITCH;
+      // implicit stencil2row of this plane (A/B buffer q & 1: last read two planes ago, before
+      // every warp passed the previous plane's barrier)
+      for (int e = tid; e < G::NE; e += W::NCW * 32) {
+        const int x = e / G::RC, y = e - (e / G::RC) * G::RC;
+        const double v = rs[x * W::TP + y];
+        const uint32_t l = sL[e];
+        sA[l & 0xffffu] = v;
+        sB[l >> 16] = v;
+      }
+      asm volatile("bar.sync 1, %0;\n" ::"n"(W::NCW * 32) : "memory");
+      const double* pa = sA + g * G::PITCH + NK * xr + t;
+      const double* pb = sB + g * G::PITCH + NK * xr + t;
+#pragma unroll
+      for (int j = 0; j < NK; ++j) {
+        const int dz = NK - 1 - j;
+        if (tc_mask & (1 << dz)) {
+#pragma unroll
+          for (int s2 = 0; s2 < KS; ++s2) {
+            dmma(acc[j][0][0], acc[j][0][1], pa[4 * s2], wa[dz][s2]);
+            dmma(acc[j][1][0], acc[j][1][1], pa[4 * s2 + NK], wa[dz][s2]);
+          }
+#pragma unroll
+          for (int s2 = 0; s2 < KS; ++s2) {
+            dmma(acc[j][0][0], acc[j][0][1], pb[4 * s2], wb[dz][s2]);
+            dmma(acc[j][1][0], acc[j][1][1], pb[4 * s2 + NK], wb[dz][s2]);
+          }
+        } else if (wz[dz] != 0.0) {
+          // centre tap of output (xr + h, g*SW + 2t + e) is region (xr + h + R, g*SW + 2t + e + R)
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const double* px = rs + (xr + h + R) * W::TP + g * G::SW + 2 * t + R;
+            acc[j][h][0] = fma(wz[dz], px[0], acc[j][h][0]);
+            acc[j][h][1] = fma(wz[dz], px[1], acc[j][h][1]);
+          }
+        }
+      }
+      __syncwarp();
+      if (lane == 0) s2r_mbar_arrive(&empty[s]);  // raw plane no longer read by this warp
+      const int64_t zo = zi - R;
+      if (zo >= z0) {
+        double* plane = a.dst.p + zo * a.dst.s0;
+        const int64_t row = (int64_t)ty * G::BM + xr;
+        if (row < a.E1) store_pair(plane + row * a.dst.s1, col, a.E2, v0, v1, acc[0][0][0], acc[0][0][1]);
+        if (row + 1 < a.E1)
+          store_pair(plane + (row + 1) * a.dst.s1, col, a.E2, v0, v1, acc[0][1][0], acc[0][1][1]);
+      }
+#pragma unroll
+      for (int j = 0; j + 1 < NK; ++j) {
+        acc[j][0][0] = acc[j + 1][0][0]; acc[j][0][1] = acc[j + 1][0][1];
+        acc[j][1][0] = acc[j + 1][1][0]; acc[j][1][1] = acc[j + 1][1][1];
+      }
+      acc[NK - 1][0][0] = acc[NK - 1][0][1] = acc[NK - 1][1][0] = acc[NK - 1][1][1] = 0.0;
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------
 int64_t persistent_grid(int occ, int max_ctas, int64_t items) {
   int64_t grid = (int64_t)(occ < 1 ? 1 : occ) * num_sms();
   if (max_ctas > 0 && grid > max_ctas) grid = max_ctas;
@@ -759,6 +902,17 @@ cudaError_t launch_s2r(int ndim, int nk, int nf, const S2RArgs& a, int tc_mask, 
       case 5: return launch_s2r2d_var<5>(a, a.s2r_variant, st);
       case 7: return launch_s2r2d_var<7>(a, a.s2r_variant, st);
     }
+  } else if (nk == 3 && s2r_ws()) {
+    using W = S2R3DWS<3>;
+    auto kern = k_s2r3d_ws<3>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, W::SMEM);
+    if (e != cudaSuccess) return e;
+    int occ = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, W::NT, W::SMEM);
+    if (e != cudaSuccess) return e;
+    const int64_t grid = persistent_grid(occ, a.max_ctas, a.ntiles);
+    kern<<<(unsigned)grid, W::NT, W::SMEM, st>>>(a, tc_mask);
+    return cudaGetLastError();
   } else if (nk == 3) {
     auto kern = k_s2r3d<3>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
