@@ -1044,7 +1044,7 @@ static cudaError_t launch_tile3d_tb(S2RArgs a, int tc_mask, cudaStream_t st) {
 //                      k-2 .. k, stored to global memory
 // Heat-3D 512^3: 313 GSt/s (round-1 k_tile3d_tb 215, Tf = 1 k_tile3d 293).  FIXED: both levels
 // hold the frame (no band fix-up).
-template <int IN_ = 4, int L1S_ = 5, int WIDE_ = 1, int NL1_ = 9>
+template <int IN_ = 4, int L1S_ = 5, int WIDE_ = 1>
 struct Tile3DTB2 {
   static constexpr int R = 1, A = 4, B = 2, KR = 6, KS = 6, H = 2, ZCH = 32;
   // WIDE = 1: 32 x 64 output tile, step-1 plane 36 x 80 (level-1 warps: 5 DMMA tiles each),
@@ -1055,12 +1055,7 @@ struct Tile3DTB2 {
   static constexpr int WIDE = WIDE_, OFF = WIDE_;
   static constexpr int BM = 32, BN = WIDE_ ? 64 : 62;   // output tile (stored)
   static constexpr int W1 = WIDE_ ? 5 : 4;               // level-1 DMMA tiles per warp
-  // level-2 / level-1 warps.  NL1 = 9: level-1 warp w computes the row of W1 tiles at rows
-  // 4w .. 4w + 3; NL1 > 9 (WIDE only): the 45 level-1 tiles are dealt round-robin, at most
-  // ceil(45 / NL1) per warp (12 warps: 4, the level-2 count)
-  static constexpr int NL2 = 8, NL1 = NL1_;
-  static constexpr int L1T = 9 * W1;                     // level-1 DMMA tiles per plane
-  static constexpr int L1PW = (L1T + NL1 - 1) / NL1;     // ... per level-1 warp (spread)
+  static constexpr int NL2 = 8, NL1 = 9;                 // level-2 / level-1 warps
   static constexpr int NT = 32 * (NL2 + NL1 + 1);
   static constexpr int TP = WIDE_ ? 84 : 68;             // plane pitch (input and step-1)
   static constexpr int RIN = 38, R1 = 36;                // staged input rows, step-1 rows
@@ -1107,41 +1102,6 @@ __device__ __forceinline__ void tb_hwindow(double (&acc)[G][2], const double* co
         }
         acc[j][0] = fma(wz[dz], v0, acc[j][0]);
         acc[j][1] = fma(wz[dz], v1, acc[j][1]);
-      }
-    }
-  }
-}
-
-// G DMMA tiles at arbitrary positions (tile index u -> rows 4 (u / W1), cols 16 (u % W1)) of the
-// level-1 step-1 plane; tiles j >= nv are skipped (warp-uniform).  Same arithmetic as tb_hwindow.
-template <class C, int G, bool ONE>
-__device__ __forceinline__ void tb_lwindow(double (&acc)[G][2], const double* const (&pl)[3], const int (&u)[G],
-                                           int nv, int tc_mask, const double (&wf)[ONE ? 1 : 3][6],
-                                           const double (&wz)[3], int lane) {
-  const int g = lane >> 2, t = lane & 3;
-  const int alpha = (2 * t) / C::B, beta = (2 * t) % C::B;
-#pragma unroll
-  for (int j = 0; j < G; ++j) acc[j][0] = acc[j][1] = 0.0;
-  int off[G];
-#pragma unroll
-  for (int j = 0; j < G; ++j) off[j] = 4 * (u[j] / C::W1) * C::TP + 16 * (u[j] % C::W1);
-#pragma unroll
-  for (int dz = 0; dz < 3; ++dz) {
-    if (tc_mask & (1 << dz)) {
-      const double* base = pl[dz] + C::OFF + C::B * g + t;
-#pragma unroll
-      for (int rho = 0; rho < C::KR; ++rho)
-#pragma unroll
-        for (int j = 0; j < G; ++j)
-          if (j < nv) dmma_t(acc[j][0], acc[j][1], base[off[j] + rho * C::TP], wf[ONE ? 0 : dz][rho]);
-    } else if (wz[dz] != 0.0) {
-#pragma unroll
-      for (int j = 0; j < G; ++j) {
-        if (j >= nv) continue;
-        const double* v = pl[dz] + off[j] + (alpha + C::R) * C::TP + C::B * g + beta + C::R + C::OFF;
-        const double2 w2 = *reinterpret_cast<const double2*>(v);  // (OFF = 1: even column)
-        acc[j][0] = fma(wz[dz], w2.x, acc[j][0]);
-        acc[j][1] = fma(wz[dz], w2.y, acc[j][1]);
       }
     }
   }
@@ -1208,7 +1168,7 @@ __global__ void __launch_bounds__(D::NT, 1)
   const bool fixed = a.hold_frame != 0;
   if (warp >= D::NL2) {
     // ---------------- level 1: step-1 planes ----------------
-    const int rb = warp - D::NL2;  // level-1 warp index (NL1 = 9: step-1 rows 4 rb .. 4 rb + 3)
+    const int rb = warp - D::NL2;  // step-1 rows 4 rb .. 4 rb + 3, cols 0 .. 16 W1 - 1
     int q = 0, p = 0;              // input / step-1 plane sequence numbers
     for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
       const int zcl = (int)(item / ncol), tile = (int)(item - (int64_t)zcl * ncol);
@@ -1231,29 +1191,13 @@ __global__ void __launch_bounds__(D::NT, 1)
         if (nl > 0) mbar_wait(&l1_empty[sl], (uint32_t)((nl - 1) & 1));
         const double* pin[3] = {in_slot(q0 + j), in_slot(q0 + j + 1), in_slot(q0 + j + 2)};
         double* dl1 = l1 + sl * D::SL1_A;
-        constexpr bool SPREAD = D::NL1 > 9;
-        constexpr int NJ = SPREAD ? D::L1PW : D::W1;
-        double acc[NJ][2];
-        int tu[NJ];
-        int nv = NJ;
-        if constexpr (SPREAD) {
-#pragma unroll
-          for (int jj = 0; jj < NJ; ++jj) tu[jj] = rb + D::NL1 * jj;
-          nv = 0;
-#pragma unroll
-          for (int jj = 0; jj < NJ; ++jj) nv += tu[jj] < D::L1T;
-          tb_lwindow<D, NJ, ONE>(acc, pin, tu, nv, tc_mask, wf, wz, lane);
-        } else {
-#pragma unroll
-          for (int jj = 0; jj < NJ; ++jj) tu[jj] = rb * D::W1 + jj;
-          tb_hwindow<D, NJ, ONE>(acc, pin, 4 * rb, 0, tc_mask, wf, wz, lane);
-        }
+        double acc[D::W1][2];
+        tb_hwindow<D, D::W1, ONE>(acc, pin, 4 * rb, 0, tc_mask, wf, wz, lane);
         const int64_t gz1 = k + a.gorg0;
         const bool zf1 = fixed && (gz1 < 1 || gz1 >= a.GE0 - 1);
 #pragma unroll
-        for (int jj = 0; jj < NJ; ++jj) {
-          if (jj >= nv) continue;
-          const int r = 4 * (tu[jj] / D::W1) + alpha, c = 16 * (tu[jj] % D::W1) + D::B * g + beta;  // step-1 coords
+        for (int jj = 0; jj < D::W1; ++jj) {
+          const int r = 4 * rb + alpha, c = 16 * jj + D::B * g + beta;  // step-1 plane coords
           double v0 = acc[jj][0], v1 = acc[jj][1];
           if (fixed && (zf1 || tile_edge)) {  // held frame points keep the input value
             const int64_t gy = sy0 + r, gx = sx0 + c;
@@ -1693,7 +1637,6 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
       if (e && e[0] == '1') return launch_tile3d_tb<Tile3DTB>(a, a.tc_mask, st);
       const char* r = getenv("CSX_TB_GEOM");  // 0: the 32 x 62 tile (equal level work)
       if (r && r[0] == '0') return launch_tile3d_tb2<Tile3DTB2<5, 6, 0>>(a, a.tc_mask, st);
-      if (r && r[0] == '2') return launch_tile3d_tb2<Tile3DTB2<4, 5, 1, 12>>(a, a.tc_mask, st);
       return launch_tile3d_tb2<Tile3DTB2<4, 5, 1>>(a, a.tc_mask, st);
     }
     if (nk == 5 || nk == 7) {
