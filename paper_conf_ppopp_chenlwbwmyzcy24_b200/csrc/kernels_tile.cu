@@ -484,6 +484,11 @@ using Tile5b = TileCfg<5, 2, 4, 8, 8, 8, 2, 2>;
 using Tile7b = TileCfg<7, 4, 2, 8, 8, 4, 4, 2>;
 using Tile3c = TileCfg<3, 4, 2, 4, 4, 6, 2, 3, 2>;
 using Tile5c = TileCfg<5, 2, 4, 8, 4, 12, 1, 3, 2>;
+// nk = 5: Tile5b with the k-slice-outer DMMA order (the default); experiments (CSX_TILE_VARIANT
+// 7 / 8): 2 CTAs / SM of 8 DMMA warps (64 x 64), row-outer and k-slice-outer (both slower)
+using Tile5bk = TileCfg<5, 2, 4, 8, 8, 8, 2, 2, 1, 1, 1>;
+using Tile5d = TileCfg<5, 2, 4, 8, 8, 4, 2, 3, 1, 2, 0>;
+using Tile5dk = TileCfg<5, 2, 4, 8, 8, 4, 2, 3, 1, 2, 1>;
 using Tile7c = TileCfg<7, 4, 2, 8, 4, 6, 2, 3, 2>;
 using Tile7d = TileCfg<7, 4, 2, 8, 8, 2, 3, 3, 1, 2>;  // variant 3: 2 CTAs/SM of 6 DMMA warps (64 x 48)
 using Tile7e = TileCfg<7, 4, 2, 8, 8, 2, 4, 2, 1, 2>;  // variant 4: 2 CTAs/SM of 8 DMMA warps (64 x 64)
@@ -1678,7 +1683,12 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
   const int v = tile_variant();
   switch (nk) {
     case 3: return v == 2 ? launch_tile_cfg<Tile3c>(a, st) : v ? launch_tile_cfg<Tile3b>(a, st) : launch_tile_cfg<Tile3>(a, st);
-    case 5: return v == 2 ? launch_tile_cfg<Tile5c>(a, st) : v ? launch_tile_cfg<Tile5b>(a, st) : launch_tile_cfg<Tile5>(a, st);
+    case 5:  // default (1): Tile5b in k-slice-outer order (Box-2D25P 311 -> 319 GSt/s); 6: Tile5b
+      if (v == 1) return launch_tile_cfg<Tile5bk>(a, st);
+      if (v == 6) return launch_tile_cfg<Tile5b>(a, st);
+      if (v == 7) return launch_tile_cfg<Tile5d>(a, st);
+      if (v == 8) return launch_tile_cfg<Tile5dk>(a, st);
+      return v == 2 ? launch_tile_cfg<Tile5c>(a, st) : launch_tile_cfg<Tile5>(a, st);
     case 9: return launch_tile_cfg<Tile9>(a, st);
     case 11: return launch_tile_cfg<Tile11>(a, st);
     case 13: return launch_tile_cfg<Tile13>(a, st);

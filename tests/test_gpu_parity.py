@@ -636,3 +636,43 @@ def test_direct_comparator_1d_variants(v, pf):
                          capture_output=True, text=True, timeout=300)
     assert out.returncode == 0, out.stderr[-2000:]
     assert float(out.stdout.strip().splitlines()[-1]) <= TOL, (v, pf, out.stdout)
+
+
+_TILE2D_SCRIPT = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+import oracle, synth
+import paper_conf_ppopp_chenlwbwmyzcy24_b200 as csx
+worst = 0.0
+for name, tf, T in (("box2d9p", 1, 3), ("box2d9p", 2, 5), ("box2d9p", 3, 7), ("box2d25p", 1, 3), ("heat2d", 2, 4)):
+    s = synth.SHAPES[name]
+    w = synth.random_weights(name)
+    u0 = synth.grid((301, 261), seed=71)
+    for bc in ("fixed", "periodic"):
+        p = csx.Plan(u0.shape, w, shape=s.kind, bc=bc, fuse_steps=tf, engine="tc_tile")
+        p.set_max_ctas(5)
+        d_in = torch.from_numpy(u0).cuda()
+        d_out = torch.empty_like(d_in)
+        p.run(d_in, d_out, T)
+        torch.cuda.synchronize()
+        ref = oracle.run(u0, w, bc, T)
+        worst = max(worst, float(np.max(np.abs(d_out.cpu().numpy() - ref)) / np.max(np.abs(ref))))
+        p.close()
+print(worst)
+"""
+
+
+@pytest.mark.parametrize("variant", ["0", "2", "3", "4", "5", "6", "7", "8"])
+def test_tile2d_variants(variant):
+    """Every 2D TC_TILE CTA geometry / DMMA order (CSX_TILE_VARIANT, read once per process: a
+    subprocess each; variant 1 is the default the rest of the suite runs) for nk = 3, 5, 7,
+    ragged tiles, both boundaries, persistent grid capped at 5 CTAs."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, "-c", _TILE2D_SCRIPT, root],
+                         env=dict(os.environ, CSX_TILE_VARIANT=variant), cwd=root,
+                         capture_output=True, text=True, timeout=300)
+    assert out.returncode == 0, out.stderr[-2000:]
+    assert float(out.stdout.strip().splitlines()[-1]) <= TOL, (variant, out.stdout)
