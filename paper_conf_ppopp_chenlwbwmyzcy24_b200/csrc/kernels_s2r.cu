@@ -577,10 +577,13 @@ __global__ void __launch_bounds__(128, 3) k_s2r3d(S2RArgs a, int tc_mask) {
     const int64_t z1 = min(a.E0, z0 + G::ZCHUNK);
     (void)nz;
     const double* base2 = a.src.p + (int64_t)(ty * G::BM - R) * a.src.s1 + (tx * G::BN - R);
-    double acc[NK][2][2];
+    constexpr int RW = G::BM / 4;  // output rows per warp (4 compute warps)
+    double acc[NK][RW][2];
 #pragma unroll
-    for (int j = 0; j < NK; ++j) acc[j][0][0] = acc[j][0][1] = acc[j][1][0] = acc[j][1][1] = 0.0;
-    const int xr = warp * 2;
+    for (int j = 0; j < NK; ++j)
+#pragma unroll
+      for (int h = 0; h < RW; ++h) acc[j][h][0] = acc[j][h][1] = 0.0;
+    const int xr = warp * RW;
     const int64_t col = (int64_t)tx * G::BN + g * G::SW + 2 * t;
     for (int64_t zi = z0 - R; zi < z1 + R; ++zi) {
       const double* base = base2 + zi * a.src.s0;
@@ -602,18 +605,18 @@ __global__ void __launch_bounds__(128, 3) k_s2r3d(S2RArgs a, int tc_mask) {
         if (tc_mask & (1 << dz)) {
 #pragma unroll
           for (int s = 0; s < KS; ++s) {
-            dmma(acc[j][0][0], acc[j][0][1], pa[4 * s], wa[dz][s]);
-            dmma(acc[j][1][0], acc[j][1][1], pa[4 * s + NK], wa[dz][s]);
+#pragma unroll
+            for (int h = 0; h < RW; ++h) dmma(acc[j][h][0], acc[j][h][1], pa[4 * s + h * NK], wa[dz][s]);
           }
 #pragma unroll
           for (int s = 0; s < KS; ++s) {
-            dmma(acc[j][0][0], acc[j][0][1], pb[4 * s], wb[dz][s]);
-            dmma(acc[j][1][0], acc[j][1][1], pb[4 * s + NK], wb[dz][s]);
+#pragma unroll
+            for (int h = 0; h < RW; ++h) dmma(acc[j][h][0], acc[j][h][1], pb[4 * s + h * NK], wb[dz][s]);
           }
         } else if (wz[dz] != 0.0) {
           // centre tap of output (xr + h, g*SW + 2t + e) is region (xr + h + R, g*SW + 2t + e + R)
 #pragma unroll
-          for (int h = 0; h < 2; ++h) {
+          for (int h = 0; h < RW; ++h) {
             const double* px = sX + (xr + h + R) * G::RC + g * G::SW + 2 * t + R;
             acc[j][h][0] = fma(wz[dz], px[0], acc[j][h][0]);
             acc[j][h][1] = fma(wz[dz], px[1], acc[j][h][1]);
@@ -624,16 +627,21 @@ __global__ void __launch_bounds__(128, 3) k_s2r3d(S2RArgs a, int tc_mask) {
       if (zo >= z0) {
         double* plane = a.dst.p + zo * a.dst.s0;
         const int64_t row = (int64_t)ty * G::BM + xr;
-        if (row < a.E1) store_pair(plane + row * a.dst.s1, col, a.E2, v0, v1, acc[0][0][0], acc[0][0][1]);
-        if (row + 1 < a.E1)
-          store_pair(plane + (row + 1) * a.dst.s1, col, a.E2, v0, v1, acc[0][1][0], acc[0][1][1]);
+#pragma unroll
+        for (int h = 0; h < RW; ++h)
+          if (row + h < a.E1)
+            store_pair(plane + (row + h) * a.dst.s1, col, a.E2, v0, v1, acc[0][h][0], acc[0][h][1]);
       }
 #pragma unroll
       for (int j = 0; j + 1 < NK; ++j) {
-        acc[j][0][0] = acc[j + 1][0][0]; acc[j][0][1] = acc[j + 1][0][1];
-        acc[j][1][0] = acc[j + 1][1][0]; acc[j][1][1] = acc[j + 1][1][1];
+#pragma unroll
+        for (int h = 0; h < RW; ++h) {
+          acc[j][h][0] = acc[j + 1][h][0];
+          acc[j][h][1] = acc[j + 1][h][1];
+        }
       }
-      acc[NK - 1][0][0] = acc[NK - 1][0][1] = acc[NK - 1][1][0] = acc[NK - 1][1][1] = 0.0;
+#pragma unroll
+      for (int h = 0; h < RW; ++h) acc[NK - 1][h][0] = acc[NK - 1][h][1] = 0.0;
     }
   }
 }
@@ -714,10 +722,13 @@ __global__ void __launch_bounds__(S2R3DWS<NK>::NT, 3) k_s2r3d_ws(S2RArgs a, int 
     const int64_t zc = item / ncol, tile = item - zc * ncol;
     const int ty = (int)(tile / a.tiles_x), tx = (int)(tile - (int64_t)ty * a.tiles_x);
     const int64_t z0 = zc * G::ZCHUNK, z1 = min(a.E0, z0 + G::ZCHUNK);
-    double acc[NK][2][2];
+    constexpr int RW = G::BM / 4;  // output rows per warp (4 compute warps)
+    double acc[NK][RW][2];
 #pragma unroll
-    for (int j = 0; j < NK; ++j) acc[j][0][0] = acc[j][0][1] = acc[j][1][0] = acc[j][1][1] = 0.0;
-    const int xr = warp * 2;
+    for (int j = 0; j < NK; ++j)
+#pragma unroll
+      for (int h = 0; h < RW; ++h) acc[j][h][0] = acc[j][h][1] = 0.0;
+    const int xr = warp * RW;
     const int64_t col = (int64_t)tx * G::BN + g * G::SW + 2 * t;
     for (int64_t zi = z0 - R; zi < z1 + R; ++zi, ++q) {
       const int s = q % W::STAGES;
@@ -743,18 +754,18 @@ __global__ void __launch_bounds__(S2R3DWS<NK>::NT, 3) k_s2r3d_ws(S2RArgs a, int 
         if (tc_mask & (1 << dz)) {
 #pragma unroll
           for (int s2 = 0; s2 < KS; ++s2) {
-            dmma(acc[j][0][0], acc[j][0][1], pa[4 * s2], wa[dz][s2]);
-            dmma(acc[j][1][0], acc[j][1][1], pa[4 * s2 + NK], wa[dz][s2]);
+#pragma unroll
+            for (int h = 0; h < RW; ++h) dmma(acc[j][h][0], acc[j][h][1], pa[4 * s2 + h * NK], wa[dz][s2]);
           }
 #pragma unroll
           for (int s2 = 0; s2 < KS; ++s2) {
-            dmma(acc[j][0][0], acc[j][0][1], pb[4 * s2], wb[dz][s2]);
-            dmma(acc[j][1][0], acc[j][1][1], pb[4 * s2 + NK], wb[dz][s2]);
+#pragma unroll
+            for (int h = 0; h < RW; ++h) dmma(acc[j][h][0], acc[j][h][1], pb[4 * s2 + h * NK], wb[dz][s2]);
           }
         } else if (wz[dz] != 0.0) {
           // centre tap of output (xr + h, g*SW + 2t + e) is region (xr + h + R, g*SW + 2t + e + R)
 #pragma unroll
-          for (int h = 0; h < 2; ++h) {
+          for (int h = 0; h < RW; ++h) {
             const double* px = rs + (xr + h + R) * W::TP + g * G::SW + 2 * t + R;
             acc[j][h][0] = fma(wz[dz], px[0], acc[j][h][0]);
             acc[j][h][1] = fma(wz[dz], px[1], acc[j][h][1]);
@@ -767,16 +778,21 @@ __global__ void __launch_bounds__(S2R3DWS<NK>::NT, 3) k_s2r3d_ws(S2RArgs a, int 
       if (zo >= z0) {
         double* plane = a.dst.p + zo * a.dst.s0;
         const int64_t row = (int64_t)ty * G::BM + xr;
-        if (row < a.E1) store_pair(plane + row * a.dst.s1, col, a.E2, v0, v1, acc[0][0][0], acc[0][0][1]);
-        if (row + 1 < a.E1)
-          store_pair(plane + (row + 1) * a.dst.s1, col, a.E2, v0, v1, acc[0][1][0], acc[0][1][1]);
+#pragma unroll
+        for (int h = 0; h < RW; ++h)
+          if (row + h < a.E1)
+            store_pair(plane + (row + h) * a.dst.s1, col, a.E2, v0, v1, acc[0][h][0], acc[0][h][1]);
       }
 #pragma unroll
       for (int j = 0; j + 1 < NK; ++j) {
-        acc[j][0][0] = acc[j + 1][0][0]; acc[j][0][1] = acc[j + 1][0][1];
-        acc[j][1][0] = acc[j + 1][1][0]; acc[j][1][1] = acc[j + 1][1][1];
+#pragma unroll
+        for (int h = 0; h < RW; ++h) {
+          acc[j][h][0] = acc[j + 1][h][0];
+          acc[j][h][1] = acc[j + 1][h][1];
+        }
       }
-      acc[NK - 1][0][0] = acc[NK - 1][0][1] = acc[NK - 1][1][0] = acc[NK - 1][1][1] = 0.0;
+#pragma unroll
+      for (int h = 0; h < RW; ++h) acc[NK - 1][h][0] = acc[NK - 1][h][1] = 0.0;
     }
   }
 }

@@ -59,11 +59,14 @@ struct S2R1D {
   static constexpr int SMEM = 2 * (STRIPS + 1) * PITCH * 8 + NE * 8;
 };
 
+#ifndef S2R3D_BM
+#define S2R3D_BM 16  // round 2: 16 (4 rows per warp); round 1 / Table 4's 8 x 64 block: 8
+#endif
 template <int NK>
 struct S2R3D {
   static constexpr int SW = NK + 1;
   static constexpr int KS = (NK * NK + 3) / 4;
-  static constexpr int BM = 8;                 // Table 4: 3D block 8 x 64
+  static constexpr int BM = S2R3D_BM;         // rows per CTA tile (4 warps x BM / 4 rows)
   static constexpr int BN = 8 * SW;
   static constexpr int RR = BM + NK - 1;
   static constexpr int RC = BN + NK - 1;
@@ -71,7 +74,7 @@ struct S2R3D {
   static constexpr int STRIPS = 8;
   static constexpr int PITCH = s2r_pitch(NK * RR);
   static constexpr int R = (NK - 1) / 2;
-  static constexpr int NT = 128;               // 4 warps x 2 output rows
+  static constexpr int NT = 128;               // 4 warps x BM / 4 output rows
   static constexpr int ZCHUNK = 64;            // output planes per work item
   static constexpr int SMEM = 2 * (STRIPS + 1) * PITCH * 8 + NE * 8 + RR * RC * 8;
 };
