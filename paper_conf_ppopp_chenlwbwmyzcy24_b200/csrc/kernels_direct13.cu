@@ -198,7 +198,10 @@ struct D3Cfg {
   static constexpr int LP = (R + 1) & ~1;  // left pad (even): staged col 0 = x0 - LP
   static constexpr int PW = BX + 2 * LP;   // staged row length (doubles, even)
   static constexpr int RY = BY + 2 * R;    // staged rows
-  static constexpr int NS = 2 * R + 2;     // ring slots: 2R+1 planes in use + 1 in flight
+  // planes in flight ahead of the window (2 measured slower at r = 1: 5 ring slots leave 2 CTAs
+  // per SM instead of 3 -- Heat-3D 220 vs 244 GSt/s)
+  static constexpr int PF = 1;
+  static constexpr int NS = 2 * R + 1 + PF;  // ring slots: 2R+1 planes in use + PF in flight
   static constexpr int PLANE = RY * PW;
   static constexpr int SMEM = NS * PLANE * 8;
   static constexpr int ZC = 32;            // output planes per work item
@@ -213,6 +216,8 @@ __device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
 }
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
+template <int K>
+__device__ __forceinline__ void cp_async_wait_n() { asm volatile("cp.async.wait_group %0;\n" ::"n"(K) : "memory"); }
 
 template <int R>
 __device__ __forceinline__ void d3_issue_plane(const DirectArgs& a, double* slot, int64_t zi,
@@ -242,9 +247,13 @@ __global__ void __launch_bounds__(256) k_direct3d(DirectArgs a, const __grid_con
     const int ty = tile / tiles_x, tx = tile - ty * tiles_x;
     const int64_t y0 = (int64_t)ty * C::BY, x0 = (int64_t)tx * C::BX;
     const int64_t z0 = zc * C::ZC, z1 = min(a.E[0], z0 + C::ZC);
-    // prologue: planes z0-R .. z0+R (slots by plane index mod NS)
-    for (int64_t zi = z0 - R; zi <= z0 + R; ++zi)
-      d3_issue_plane<R>(a, sm + (int)((zi + 2 * C::NS) % C::NS) * C::PLANE, zi, y0, x0);
+    // prologue: planes z0-R .. z0+R+PF-1 (slots by plane index mod NS), one commit group each
+    // (a group past the chunk's last plane z1+R-1 is committed empty, so that the number of
+    // groups per plane stays one and wait_group<PF - 1> always means "window complete")
+    for (int64_t zi = z0 - R; zi <= z0 + R + C::PF - 1; ++zi) {
+      if (zi < z1 + R) d3_issue_plane<R>(a, sm + (int)((zi + 2 * C::NS) % C::NS) * C::PLANE, zi, y0, x0);
+      else cp_async_commit();
+    }
     // this thread's outputs: rows y0 + 4 warp + j (j < 4), cols x0 + 2 lane + e
     const int ry = 4 * warp, cx = 2 * lane;
     const int64_t gy0 = a.gorg[1] + y0 + ry, gx0 = a.gorg[2] + x0 + cx;
@@ -252,10 +261,13 @@ __global__ void __launch_bounds__(256) k_direct3d(DirectArgs a, const __grid_con
       // planes up to zo+R have landed (this thread's copies), then everyone's (barrier); the
       // barrier also retires iteration zo-1, the last reader of plane zo-R-1, whose slot now
       // receives plane zo+R+1 while output plane zo is computed
-      cp_async_wait_all();
+      cp_async_wait_n<C::PF - 1>();
       __syncthreads();
-      if (zo + 1 < z1)
-        d3_issue_plane<R>(a, sm + (int)((zo + R + 1 + 2 * C::NS) % C::NS) * C::PLANE, zo + R + 1, y0, x0);
+      {
+        const int64_t zn = zo + R + C::PF;  // its slot held plane zo-R-1, read last iteration
+        if (zn < z1 + R) d3_issue_plane<R>(a, sm + (int)((zn + 2 * C::NS) % C::NS) * C::PLANE, zn, y0, x0);
+        else cp_async_commit();
+      }
       double acc[4][2];
 #pragma unroll
       for (int j = 0; j < 4; ++j) acc[j][0] = acc[j][1] = 0.0;

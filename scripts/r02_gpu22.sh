@@ -1,0 +1,7 @@
+#!/bin/bash
+OUT=gpurun_out/r02ap; mkdir -p $OUT
+timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_coverage.py -q -k "direct" > $OUT/t.log 2>&1; echo "rc=$?" >> $OUT/t.log
+B="python bench.py --steps 5 --warmup 3 --no-cpu-baseline --no-e2e --no-comparator --engine direct"
+for c in heat3d_512 box3d27p_512 star3d13p_512 box3d125p_512; do
+  echo "$c $(timeout 300 $B --config $c 2>/dev/null)" >> $OUT/sweep.txt
+done
