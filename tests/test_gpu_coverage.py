@@ -251,3 +251,48 @@ def test_parity_3d_general_radius_variants(csx, monkeypatch, env):
         for bc in ("fixed", "periodic"):
             got, _ = run_gpu(csx, u0, w, s.kind, bc, 2, engine="tc_tile", max_ctas=5)
             assert rel(got, oracle.run(u0, w, bc, 2)) <= TOL, (name, bc, env)
+
+
+def test_randomized_plans_against_oracle(csx):
+    """Seeded fuzzing over the plan space the C-ABI accepts: dimension, radius, star / box,
+    signed weights, ragged extents (including extents equal to the composed window), boundary,
+    fusion depth, engine, T with and without a remainder, persistent-grid caps, in place or not.
+    Every run is compared element by element with the oracle; refusals must be UNSUPPORTED."""
+    rng = np.random.default_rng(20241017)
+    ran = 0
+    for case in range(200):
+        ndim = int(rng.integers(1, 4))
+        r = int(rng.integers(1, 4))
+        box = bool(rng.integers(0, 2)) or ndim == 1
+        maxtf = {1: 15 // r, 2: 6 // r, 3: 2 if r == 1 else 1}[ndim]
+        tf = int(rng.integers(1, max(1, maxtf) + 1))
+        nk = 2 * r * tf + 1
+        if ndim == 1:
+            ext = (int(rng.integers(nk, 9000)),)
+        elif ndim == 2:
+            ext = tuple(int(rng.integers(nk, 300)) for _ in range(2))
+        else:
+            ext = tuple(int(rng.integers(nk, 60)) for _ in range(3))
+        bc = ("fixed", "periodic")[int(rng.integers(0, 2))]
+        engine = ("auto", "tc_tile", "tc_s2r", "direct")[int(rng.integers(0, 4))]
+        T = int(rng.integers(1, 3 * tf + 2))
+        cap = int((0, 0, 1, 3, 7)[int(rng.integers(0, 5))])
+        w = synth.random_signed_weights(ndim, r, seed=1000 + case, box=box)
+        u0 = synth.grid(ext, seed=2000 + case)
+        try:
+            p = csx.Plan(ext, w, shape="box" if box else "star", bc=bc, fuse_steps=tf, engine=engine)
+        except csx.CsxError as e:
+            assert e.status == csx.CSX_ERR_UNSUPPORTED, (case, ndim, r, tf, engine, str(e))
+            continue
+        if cap:
+            p.set_max_ctas(cap)
+        d_in = torch.from_numpy(u0).cuda()
+        d_out = d_in if rng.integers(0, 4) == 0 else torch.empty_like(d_in)
+        p.run(d_in, d_out, T)
+        torch.cuda.synchronize()
+        got = d_out.cpu().numpy()
+        p.close()
+        ref = oracle.run(u0, w, bc, T)
+        assert rel(got, ref) <= TOL, (case, ndim, r, box, tf, ext, bc, engine, T, cap)
+        ran += 1
+    assert ran >= 120, ran
