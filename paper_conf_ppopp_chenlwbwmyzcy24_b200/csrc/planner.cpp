@@ -329,12 +329,14 @@ int auto_tf(int ndim, int radius, int engine) {
   // DESIGN.md "Fusion depth" (reading A4): 2D r=1 -> 3 (the paper's Box-2D9P choice,
   // P.1478-1480); r >= 2 in 2D and all 3D -> 1 (one N fragment, lowest DMMA count per
   // point-step on B200).  1D is HBM-bound, so deeper fusion pays until the DMMA work of the
-  // Toeplitz blocks (K = nk + 7) meets the HBM time: TC_TILE takes nk ~ 19..23 (r=1 -> 11,
-  // r=2 -> 5, r=3 -> 3; measured sweep in DESIGN.md §12); TC_S2R's paper layout keeps
-  // nk + 1 <= 16 (two N fragments): r=1 -> 7, r=2 -> 3, r=3 -> 2.
+  // Toeplitz blocks (K = nk + 7) meets the HBM time: TC_TILE takes nk ~ 27..29 (r=1 -> 13,
+  // r=2 -> 7, r=3 -> 3; round-2 sweep on Heat-1D / 1D5P, 10.24M and 102.4M points: Tf 9 / 11 /
+  // 13 / 15 = 2845 / 3136 / 3263 / 3166 and 3060 / 3509 / 3877 / 4152 GSt/s; 1D5P Tf 4..7 best
+  // at 7); TC_S2R's paper layout keeps nk + 1 <= 16 (two N fragments): r=1 -> 7, r=2 -> 3,
+  // r=3 -> 2.
   if (ndim == 1) {
     if (engine == CSX_ENGINE_TC_S2R) return radius == 1 ? 7 : (radius == 2 ? 3 : 2);
-    return radius == 1 ? 11 : (radius == 2 ? 5 : 3);
+    return radius == 1 ? 13 : (radius == 2 ? 7 : 3);
   }
   // the CUDA-core comparator's own best depth: 2D r = 1 -> 4 (register wavefront, Box-2D9P
   // 10240^2: Tf 1/2/3/4 = 310 / 640 / 681 / 766 GSt/s), r >= 2 -> 1

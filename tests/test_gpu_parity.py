@@ -104,7 +104,7 @@ def test_parity_fusion_depths_1d(csx, tf):
         assert rel(got, oracle.run(u0, w, bc, 23)) <= TOL, (tf, bc)
 
 
-@pytest.mark.parametrize("r,tf", [(1, 1), (1, 3), (1, 7), (1, 8), (1, 11), (1, 15), (2, 3), (2, 5),
+@pytest.mark.parametrize("r,tf", [(1, 1), (1, 3), (1, 7), (1, 8), (1, 11), (1, 13), (1, 15), (2, 3), (2, 5),
                                   (2, 7), (3, 2), (3, 5)])
 def test_parity_fusion_depths_1d_tile(csx, r, tf):
     """TC_TILE 1D (Toeplitz blocks, nk = 2 r Tf + 1 up to 31): 3 full tiles of 8 x 256 outputs

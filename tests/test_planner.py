@@ -258,7 +258,7 @@ def test_2d_fusion_limits():
 
 def test_auto_fusion_depths():
     # (3D r = 1 stars run two steps per pass by temporal blocking; boxes and r >= 2 one)
-    cases = {"heat1d": 11, "1d5p": 5, "heat2d": 3, "box2d9p": 3, "star2d13p": 1, "box2d49p": 1,
+    cases = {"heat1d": 13, "1d5p": 7, "heat2d": 3, "box2d9p": 3, "star2d13p": 1, "box2d49p": 1,
              "heat3d": 2, "box3d27p": 1, "star3d13p": 1, "box3d125p": 1}
     for name, tf in cases.items():
         s = synth.SHAPES[name]
