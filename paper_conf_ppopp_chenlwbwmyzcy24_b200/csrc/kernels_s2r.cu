@@ -208,6 +208,9 @@ __global__ void __launch_bounds__(S2R2D<NK>::NT, 2) k_s2r2d(S2RArgs a) {
 //   warps 0 .. NCW-1    dual tessellation on DMMA from A/B buffer it % 2, centre store
 // Buffer hand-offs are mbarriers: raw full/empty, ab_full (scatter warps arrive) and ab_empty
 // (DMMA warps arrive), so tile k+1 is scattered while tile k is tessellated.
+#ifndef S2R_NG7
+#define S2R_NG7 2
+#endif
 template <int NK, bool PAD = true>
 struct S2R2DWS {
   using G = S2R2D<NK, PAD>;
@@ -217,37 +220,41 @@ struct S2R2DWS {
   // CTAs per SM with two scatter warps
   static constexpr int MINB = NK >= 7 ? 1 : 2;
   static constexpr int NSW = NK >= 7 ? 4 : 2;
+  // nk = 7 (one CTA per SM): two groups of 8 DMMA warps tessellate alternate tiles, four A/B
+  // buffers in flight (16 DMMA warps per SM as at two CTAs, without the second LUT and ring)
+  static constexpr int NG = NK >= 7 ? S2R_NG7 : 1;
+  static constexpr int NB = 2 * NG;                    // A/B buffers
   static constexpr int RAW_STAGES = 2;
-  static constexpr int NT = 32 * (G::NCW + NSW + 1);
-  static constexpr int SMEM = RAW_STAGES * G::RAW * 8 + G::AB_BUFS * G::AB * 8 + G::NE * 4;
+  static constexpr int NT = 32 * (NG * G::NCW + NSW + 1);
+  static constexpr int SMEM = RAW_STAGES * G::RAW * 8 + NB * G::AB * 8 + G::NE * 4;
 };
 
 template <int NK, bool PAD, bool DIRTY>
 __global__ void __launch_bounds__(S2R2DWS<NK>::NT, S2R2DWS<NK>::MINB) k_s2r2d_ws(S2RArgs a) {
   using G = S2R2D<NK, PAD>;
   using W = S2R2DWS<NK, PAD>;
-  constexpr int NSW = W::NSW;
+  constexpr int NSW = W::NSW, NB = W::NB, NCW = W::NG * G::NCW;
   extern __shared__ __align__(128) double smem[];
-  __shared__ __align__(8) uint64_t full[W::RAW_STAGES], empty[W::RAW_STAGES], ab_full[2], ab_empty[2];
+  __shared__ __align__(8) uint64_t full[W::RAW_STAGES], empty[W::RAW_STAGES], ab_full[NB], ab_empty[NB];
   double* raw = smem;                                           // RAW_STAGES x RAW
-  double* sAB = raw + W::RAW_STAGES * G::RAW;                   // 2 x (A | B)
-  uint32_t* sL = reinterpret_cast<uint32_t*>(sAB + G::AB_BUFS * G::AB);
+  double* sAB = raw + W::RAW_STAGES * G::RAW;                   // NB x (A | B)
+  uint32_t* sL = reinterpret_cast<uint32_t*>(sAB + NB * G::AB);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  for (int i = tid; i < G::AB_BUFS * G::AB; i += S2R2DWS<NK>::NT) sAB[i] = 0.0;
-  for (int i = tid; i < G::NE; i += S2R2DWS<NK>::NT) sL[i] = (uint32_t)a.lut[i].y;
+  for (int i = tid; i < NB * G::AB; i += W::NT) sAB[i] = 0.0;
+  for (int i = tid; i < G::NE; i += W::NT) sL[i] = (uint32_t)a.lut[i].y;
   if (tid == 0) {
     for (int s = 0; s < W::RAW_STAGES; ++s) {
       s2r_mbar_init(&full[s], 1);
       s2r_mbar_init(&empty[s], NSW);
     }
-    for (int b = 0; b < 2; ++b) {
+    for (int b = 0; b < NB; ++b) {
       s2r_mbar_init(&ab_full[b], NSW);
-      s2r_mbar_init(&ab_empty[b], G::NCW);
+      s2r_mbar_init(&ab_empty[b], G::NCW);  // one DMMA group
     }
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
   }
   __syncthreads();
-  if (warp == G::NCW + NSW) {  // producer
+  if (warp == NCW + NSW) {  // producer
     int it = 0;
     for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
       const int s = it % W::RAW_STAGES, n = it / W::RAW_STAGES;
@@ -259,12 +266,12 @@ __global__ void __launch_bounds__(S2R2DWS<NK>::NT, S2R2DWS<NK>::MINB) k_s2r2d_ws
     }
     return;
   }
-  if (warp >= G::NCW) {  // scatter warps: implicit stencil2row through the LUT (branch-free)
-    const int sw = warp - G::NCW;
+  if (warp >= NCW) {  // scatter warps: implicit stencil2row through the LUT (branch-free)
+    const int sw = warp - NCW;
     int it = 0;
     for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
-      const int s = it % W::RAW_STAGES, b = it & 1;
-      if (it >= 2) s2r_mbar_wait(&ab_empty[b], ((it >> 1) - 1) & 1);  // tile it-2 tessellated
+      const int s = it % W::RAW_STAGES, b = it % NB;
+      if (it >= NB) s2r_mbar_wait(&ab_empty[b], ((it / NB) - 1) & 1);  // tile it-NB tessellated
       s2r_mbar_wait(&full[s], (it / W::RAW_STAGES) & 1);
       double* sA = sAB + b * G::AB;
       double* sB = sA + (G::STRIPS + 1) * G::PITCH;
@@ -302,13 +309,15 @@ __global__ void __launch_bounds__(S2R2DWS<NK>::NT, S2R2DWS<NK>::MINB) k_s2r2d_ws
   const int g = lane >> 2, t = lane & 3;
   const bool v0 = 2 * t < G::SW, v1 = 2 * t + 1 < G::SW;
   constexpr int RW = G::BM / G::NCW;
-  const int xr0 = warp * RW;
+  const int grp = warp / G::NCW;              // DMMA group: tiles it with it % NG == grp
+  const int xr0 = (warp - grp * G::NCW) * RW;
   int it = 0;
   for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
-    const int b = it & 1;
+    if (it % W::NG != grp) continue;
+    const int b = it % NB;
     const int ty = (int)(tile / a.tiles_x);
     const int tx = (int)(tile - (int64_t)ty * a.tiles_x);
-    s2r_mbar_wait(&ab_full[b], (it >> 1) & 1);
+    s2r_mbar_wait(&ab_full[b], (it / NB) & 1);
     const double* sA = sAB + b * G::AB;
     const double* sB = sA + (G::STRIPS + 1) * G::PITCH;
     const double* pa = sA + g * G::PITCH + G::NKV * xr0 + t;
