@@ -103,6 +103,14 @@ __device__ __forceinline__ void st_out(double* p, double v0, double v1, bool hin
     *reinterpret_cast<double2*>(p) = make_double2(v0, v1);
 }
 
+// 8-B output store (same hint)
+__device__ __forceinline__ void st_out1(double* p, double v, bool hinted, uint64_t pol) {
+  if (hinted)
+    asm volatile("st.global.L2::cache_hint.f64 [%0], %1, %2;\n" ::"l"(p), "d"(v), "l"(pol) : "memory");
+  else
+    *p = v;
+}
+
 __device__ __forceinline__ void bulk_g2s_hint(void* dst, const void* src, uint32_t bytes, uint64_t* bar,
                                               uint64_t pol) {
   asm volatile(
@@ -520,8 +528,13 @@ static int tile_variant() {
 // window (2x4 for nk = 5, 4x2 for nk = 7: the smaller K, as in 2D) and, where NK x KS weight
 // fragments would not fit the register file (WREG = 0, nk = 7: 7 x 20), each TC plane's KS
 // fragments loaded from L1 just before its GEMM (KS loads per G*KS DMMAs).
+// TPX: extra staged columns (a row pitch whose bank offset keeps the star planes' DFMA loads
+// conflict-free); CM: column-major numbering of the a x b output block in the DMMA N dimension
+// (n -> alpha = n % a, beta = n / a, only a = 2), so a lane's two accumulators are vertically
+// adjacent and the DFMA planes load them as two conflict-free LDS.64 rows instead of one
+// 2-way-conflicted LDS.128 (round 2: 36 M smem load conflicts per Star-3D13P launch).
 template <int NK_, int G_, int WM_, int WN_, int STAGES_, int ZCH_, int CG_ = 1, int KO_ = 0,
-          int A_ = 4, int B_ = 2, int WREG_ = 1>
+          int A_ = 4, int B_ = 2, int WREG_ = 1, int TPX_ = 0, int CM_ = 0>
 struct Tile3DCfg {
   static constexpr int NK = NK_, A = A_, B = B_, KC = 4 * ((B_ + NK - 1 + 3) / 4), G = G_, WM = WM_,
                        WN = WN_, STAGES = STAGES_, ZCH = ZCH_, CG = CG_;
@@ -538,7 +551,9 @@ struct Tile3DCfg {
   static constexpr int WC = CG * 8 * B;             // output cols per warp (CG column groups)
   static constexpr int BN = WN * WC;
   static constexpr int RR = BM + NK - 1;
-  static constexpr int TP = ((ODD + BN + KC - B) + 1) / 2 * 2;
+  static constexpr int TP = ((ODD + BN + KC - B) + 1) / 2 * 2 + TPX_;
+  static constexpr int CM = CM_;
+  static_assert(!CM || (A == 2 && CG == 1), "column-major block numbering: a = 2 only");
   static constexpr int STAGE = RR * TP;
   static constexpr int STAGE_A = (STAGE + 15) / 16 * 16;  // ring slot (128-B aligned)
   static constexpr int NCW = WM * WN;
@@ -650,7 +665,22 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
 #pragma unroll
     for (int k = 0; k < C::KS; ++k) wf[0][k] = __ldg(a.frags + (dz1 * C::KS + k) * 32 + lane);
   }
-  const int alpha = (2 * t) / C::B, beta = (2 * t) % C::B;
+  // CM: B-fragment lane (k = lane % 4, n' = lane / 4) takes the planner's column n = alpha * b +
+  // beta of its output (alpha, beta) = (n' % 2, n' / 2)
+  const int cm_src = (lane & 3) + 4 * (((lane >> 2) & 1) * C::B + (lane >> 3));
+  if (C::CM) {
+    if (C::WREG) {
+#pragma unroll
+      for (int p = 0; p < C::NK; ++p)
+#pragma unroll
+        for (int k = 0; k < C::KS; ++k) wf[C::WREG ? p : 0][k] = __shfl_sync(0xffffffffu, wf[C::WREG ? p : 0][k], cm_src);
+    } else if (single_tc) {
+#pragma unroll
+      for (int k = 0; k < C::KS; ++k) wf[0][k] = __shfl_sync(0xffffffffu, wf[0][k], cm_src);
+    }
+  }
+  // this lane's accumulator e sits at block position (alpha + e * CM, beta + e * (1 - CM))
+  const int alpha = C::CM ? 0 : (2 * t) / C::B, beta = C::CM ? t : (2 * t) % C::B;
   const bool any_cuda = tc_mask != (1 << C::NK) - 1;
   uint64_t spol = 0;
   if (a.l2hint == 3) asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;\n" : "=l"(spol));
@@ -698,7 +728,10 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
         const double* stg = smem + slot[dz] * C::STAGE_A;
         if (!C::WREG && !single_tc && (tc_mask & (1 << dz))) {  // this plane's fragments, from L1
 #pragma unroll
-          for (int k = 0; k < C::KS; ++k) wf[0][k] = __ldg(a.frags + (dz * C::KS + k) * 32 + lane);
+          for (int k = 0; k < C::KS; ++k) {
+            wf[0][k] = __ldg(a.frags + (dz * C::KS + k) * 32 + lane);
+            if (C::CM) wf[0][k] = __shfl_sync(0xffffffffu, wf[0][k], cm_src);
+          }
         }
         const int wp = C::WREG ? dz : 0;
         if ((tc_mask & (1 << dz)) && C::KO == 1) {
@@ -739,9 +772,15 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
           for (int cg = 0; cg < C::CG; ++cg)
 #pragma unroll
             for (int j = 0; j < C::G; ++j) {
-              const double2 v = *reinterpret_cast<const double2*>(stg + frame_off + C::A * j * C::TP + cg * 8 * C::B);
-              acc[cg][j][0] = fma(wz[dz], v.x, acc[cg][j][0]);
-              acc[cg][j][1] = fma(wz[dz], v.y, acc[cg][j][1]);
+              if (C::CM) {  // vertically adjacent pair: two conflict-free row loads
+                const double* q = stg + frame_off + C::A * j * C::TP;
+                acc[cg][j][0] = fma(wz[dz], q[0], acc[cg][j][0]);
+                acc[cg][j][1] = fma(wz[dz], q[C::TP], acc[cg][j][1]);
+              } else {
+                const double2 v = *reinterpret_cast<const double2*>(stg + frame_off + C::A * j * C::TP + cg * 8 * C::B);
+                acc[cg][j][0] = fma(wz[dz], v.x, acc[cg][j][0]);
+                acc[cg][j][1] = fma(wz[dz], v.y, acc[cg][j][1]);
+              }
             }
         }
       }
@@ -754,9 +793,15 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
 #pragma unroll
         for (int cg = 0; cg < C::CG; ++cg)
 #pragma unroll
-          for (int j = 0; j < C::G; ++j)
-            st_out(p0 + (int64_t)(C::A * j) * a.dst.s1 + cg * 8 * C::B, acc[cg][j][0], acc[cg][j][1],
-                   a.l2hint == 3, spol);
+          for (int j = 0; j < C::G; ++j) {
+            if (C::CM) {  // rows row0 + A j and + 1: each warp store covers 32 consecutive columns
+              st_out1(p0 + (int64_t)(C::A * j) * a.dst.s1, acc[cg][j][0], a.l2hint == 3, spol);
+              st_out1(p0 + (int64_t)(C::A * j + 1) * a.dst.s1, acc[cg][j][1], a.l2hint == 3, spol);
+            } else {
+              st_out(p0 + (int64_t)(C::A * j) * a.dst.s1 + cg * 8 * C::B, acc[cg][j][0], acc[cg][j][1],
+                     a.l2hint == 3, spol);
+            }
+          }
       } else {
         const double* cstg = smem + slot[C::R] * C::STAGE_A;
         const bool edge = tile_edge || plane_frame;
@@ -764,19 +809,17 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
         for (int cg = 0; cg < C::CG; ++cg)
 #pragma unroll
           for (int j = 0; j < C::G; ++j) {
-            const int64_t row = row0 + C::A * j, col = col0 + cg * 8 * C::B;
-            if (row >= a.E1 || col >= a.E2) continue;
-            double* p = plane + row * a.dst.s1 + col;
-            const int64_t grow = row + a.gorg1;
-            const bool rf = plane_frame || grow < C::R || grow >= a.GE1 - C::R;
 #pragma unroll
             for (int e = 0; e < 2; ++e) {
-              const int64_t c = col + e, gc = c + a.gorg2;
-              if (c >= a.E2) continue;
+              const int64_t row = row0 + C::A * j + (C::CM ? e : 0);
+              const int64_t c = col0 + cg * 8 * C::B + (C::CM ? 0 : e), gc = c + a.gorg2;
+              if (row >= a.E1 || c >= a.E2) continue;
+              const int64_t grow = row + a.gorg1;
+              const bool rf = plane_frame || grow < C::R || grow >= a.GE1 - C::R;
               double v = acc[cg][j][e];
               if (edge && (rf || gc < C::R || gc >= a.GE2 - C::R))
-                v = cstg[frame_off + C::A * j * C::TP + cg * 8 * C::B + e];
-              p[e] = v;
+                v = cstg[frame_off + C::A * j * C::TP + cg * 8 * C::B + (C::CM ? e * C::TP : e)];
+              plane[row * a.dst.s1 + c] = v;
             }
           }
       }
@@ -1335,6 +1378,11 @@ using Tile3D5k = Tile3DCfg<5, 4, 4, 2, 9, 32, 1, 1, 2, 4, 0>;
 using Tile3D7k = Tile3DCfg<7, 4, 2, 4, 10, 32, 1, 1, 4, 2, 0>;
 // radius 2 with twice the blocks per warp (8 accumulator chains, CTA 64 x 64, 6-plane ring)
 using Tile3D5g = Tile3DCfg<5, 8, 4, 2, 6, 32, 1, 1, 2, 4, 0>;
+// star shapes, conflict-free DFMA planes: r = 2 with the column-major block numbering (the
+// 72-column pitch would not fit the 6-plane ring), r = 3 with a 76-column pitch (2 TP = 24 banks
+// mod 32: the four block rows of one 8-lane LDS.128 phase fall on disjoint banks)
+using Tile3D5gc = Tile3DCfg<5, 8, 4, 2, 6, 32, 1, 1, 2, 4, 0, 0, 1>;
+using Tile3D7ks = Tile3DCfg<7, 4, 2, 4, 10, 32, 1, 1, 4, 2, 0, 4>;
 
 
 // ------------------------------------------------------------------------------------------
@@ -1652,7 +1700,12 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
       // ring; Box-3D125P 59.9 vs 58.4).  CSX_TILE3D5_G8 = 0 / 1 forces either.
       const char* g8 = getenv("CSX_TILE3D5_G8");
       const bool star = __builtin_popcount((unsigned)a.tc_mask) == 1;
-      if (nk == 5 && (g8 ? g8[0] == '1' : star)) return launch_tile3d_cfg<Tile3D5g>(a, a.tc_mask, st);
+      // star: conflict-free DFMA plane loads (CSX_STAR_CF = 0: the round-2 layouts)
+      const char* cf = getenv("CSX_STAR_CF");
+      const bool scf = star && !(cf && cf[0] == '0');
+      if (nk == 5 && (g8 ? g8[0] == '1' : star))
+        return scf ? launch_tile3d_cfg<Tile3D5gc>(a, a.tc_mask, st) : launch_tile3d_cfg<Tile3D5g>(a, a.tc_mask, st);
+      if (nk == 7 && scf && ko) return launch_tile3d_cfg<Tile3D7ks>(a, a.tc_mask, st);
       if (nk == 5) return ko ? launch_tile3d_cfg<Tile3D5k>(a, a.tc_mask, st) : launch_tile3d_cfg<Tile3D5>(a, a.tc_mask, st);
       return ko ? launch_tile3d_cfg<Tile3D7k>(a, a.tc_mask, st) : launch_tile3d_cfg<Tile3D7>(a, a.tc_mask, st);
     }

@@ -101,7 +101,8 @@ CAP_CASES = [
     ("heat3d", (70, 37, 130), 3, "tc_tile", 1),   # k_tile3d nk = 3, star variant
     ("box3d27p", (70, 37, 130), 3, "tc_tile", 1),  # k_tile3d nk = 3, box variant
     ("box3d125p", (70, 37, 130), 2, "tc_tile", 1),  # k_tile3d nk = 5
-    ("star3d19p", (70, 37, 130), 2, "tc_tile", 1),  # k_tile3d nk = 7
+    ("star3d19p", (70, 37, 130), 2, "tc_tile", 1),  # k_tile3d nk = 7 (star: 76-column pitch)
+    ("star3d13p", (70, 37, 130), 2, "tc_tile", 1),  # k_tile3d nk = 5 (star: column-major blocks)
     ("heat3d", (70, 37, 130), 4, "tc_tile", 2),   # k_tile3d_tb
     ("box2d9p", (300, 260), 7, "tc_s2r", 3),      # k_s2r2d nk = 7
     ("box2d25p", (300, 260), 3, "tc_s2r", 1),     # k_s2r2d nk = 5
@@ -238,10 +239,12 @@ def test_graph_plan_variant_switch_teardown(csx):
     assert leak < (8 << 20), f"{leak >> 20} MB not returned"
 
 
-@pytest.mark.parametrize("env", [{"CSX_TILE3D_KO": "0"}, {"CSX_TILE3D5_G8": "1"}, {"CSX_TILE3D5_G8": "0"}])
+@pytest.mark.parametrize("env", [{"CSX_TILE3D_KO": "0"}, {"CSX_TILE3D5_G8": "1"}, {"CSX_TILE3D5_G8": "0"},
+                                 {"CSX_STAR_CF": "0"}])
 def test_parity_3d_general_radius_variants(csx, monkeypatch, env):
     """The other 3D r = 2 / 3 tile configurations (row-outer DMMA order; 8 or 4 blocks per warp
-    for both stars and boxes; read at every launch): ragged tiles and z chunks, both boundaries."""
+    for both stars and boxes; the round-2 star layouts without the conflict-free DFMA planes;
+    read at every launch): ragged tiles and z chunks, both boundaries."""
     for k, v in env.items():
         monkeypatch.setenv(k, v)
     for name in R3D:
