@@ -723,8 +723,57 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
       for (int cg = 0; cg < C::CG; ++cg)
 #pragma unroll
         for (int j = 0; j < C::G; ++j) acc[cg][j][0] = acc[cg][j][1] = 0.0;
+      if constexpr (C::KO == 2) {
+        // KO = 2 (box shapes, every plane on the tensor cores, weights in registers): input
+        // rows outer as in KO = 0 (one A fragment per plane and row feeds every block whose
+        // window holds the row), but the NK planes interleaved with one accumulator set each,
+        // so consecutive DMMAs belong to NK independent chains instead of one (the KO = 0
+        // schedule issued up to 5 dependent DMMAs back to back); summed at the end
+        double accz[C::NK][C::CG][C::G][2];
 #pragma unroll
-      for (int dz = 0; dz < C::NK; ++dz) {
+        for (int dz = 0; dz < C::NK; ++dz)
+#pragma unroll
+          for (int cg = 0; cg < C::CG; ++cg)
+#pragma unroll
+            for (int j = 0; j < C::G; ++j) accz[dz][cg][j][0] = accz[dz][cg][j][1] = 0.0;
+#pragma unroll
+        for (int ra = 0; ra < C::A * C::G + C::NK - 1; ++ra) {
+          double f[C::NK][C::CG][C::KC / 4];
+#pragma unroll
+          for (int dz = 0; dz < C::NK; ++dz)
+#pragma unroll
+            for (int cg = 0; cg < C::CG; ++cg)
+#pragma unroll
+              for (int h = 0; h < C::KC / 4; ++h)
+                f[dz][cg][h] = smem[slot[dz] * C::STAGE_A + lane_off + ra * C::TP + cg * 8 * C::B + 4 * h];
+#pragma unroll
+          for (int h = 0; h < C::KC / 4; ++h)
+#pragma unroll
+            for (int j = 0; j < C::G; ++j) {
+              const int rho = ra - C::A * j;
+              if (rho >= 0 && rho < C::KR)
+#pragma unroll
+                for (int dz = 0; dz < C::NK; ++dz)
+#pragma unroll
+                  for (int cg = 0; cg < C::CG; ++cg)
+                    dmma_t(accz[dz][cg][j][0], accz[dz][cg][j][1], f[dz][cg][h],
+                           wf[C::WREG ? dz : 0][rho * (C::KC / 4) + h]);
+            }
+        }
+#pragma unroll
+        for (int cg = 0; cg < C::CG; ++cg)
+#pragma unroll
+          for (int j = 0; j < C::G; ++j)
+#pragma unroll
+            for (int e = 0; e < 2; ++e) {
+              double v = accz[0][cg][j][e];
+#pragma unroll
+              for (int dz = 1; dz < C::NK; ++dz) v += accz[dz][cg][j][e];
+              acc[cg][j][e] = v;
+            }
+      }
+#pragma unroll
+      for (int dz = 0; dz < (C::KO == 2 ? 0 : C::NK); ++dz) {
         const double* stg = smem + slot[dz] * C::STAGE_A;
         if (!C::WREG && !single_tc && (tc_mask & (1 << dz))) {  // this plane's fragments, from L1
 #pragma unroll
@@ -809,17 +858,34 @@ __global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
         for (int cg = 0; cg < C::CG; ++cg)
 #pragma unroll
           for (int j = 0; j < C::G; ++j) {
+            if constexpr (C::CM) {  // accumulator e at row + e, same column
 #pragma unroll
-            for (int e = 0; e < 2; ++e) {
-              const int64_t row = row0 + C::A * j + (C::CM ? e : 0);
-              const int64_t c = col0 + cg * 8 * C::B + (C::CM ? 0 : e), gc = c + a.gorg2;
-              if (row >= a.E1 || c >= a.E2) continue;
+              for (int e = 0; e < 2; ++e) {
+                const int64_t row = row0 + C::A * j + e;
+                const int64_t c = col0 + cg * 8 * C::B, gc = c + a.gorg2;
+                if (row >= a.E1 || c >= a.E2) continue;
+                const int64_t grow = row + a.gorg1;
+                const bool rf = plane_frame || grow < C::R || grow >= a.GE1 - C::R;
+                double v = acc[cg][j][e];
+                if (edge && (rf || gc < C::R || gc >= a.GE2 - C::R))
+                  v = cstg[frame_off + (C::A * j + e) * C::TP + cg * 8 * C::B];
+                plane[row * a.dst.s1 + c] = v;
+              }
+            } else {
+              const int64_t row = row0 + C::A * j, col = col0 + cg * 8 * C::B;
+              if (row >= a.E1 || col >= a.E2) continue;
+              double* p = plane + row * a.dst.s1 + col;
               const int64_t grow = row + a.gorg1;
               const bool rf = plane_frame || grow < C::R || grow >= a.GE1 - C::R;
-              double v = acc[cg][j][e];
-              if (edge && (rf || gc < C::R || gc >= a.GE2 - C::R))
-                v = cstg[frame_off + C::A * j * C::TP + cg * 8 * C::B + (C::CM ? e * C::TP : e)];
-              plane[row * a.dst.s1 + c] = v;
+#pragma unroll
+              for (int e = 0; e < 2; ++e) {
+                const int64_t c = col + e, gc = c + a.gorg2;
+                if (c >= a.E2) continue;
+                double v = acc[cg][j][e];
+                if (edge && (rf || gc < C::R || gc >= a.GE2 - C::R))
+                  v = cstg[frame_off + C::A * j * C::TP + cg * 8 * C::B + e];
+                p[e] = v;
+              }
             }
           }
       }
@@ -1092,8 +1158,17 @@ static cudaError_t launch_tile3d_tb(S2RArgs a, int tc_mask, cudaStream_t st) {
 //                      k-2 .. k, stored to global memory
 // Heat-3D 512^3: 313 GSt/s (round-1 k_tile3d_tb 215, Tf = 1 k_tile3d 293).  FIXED: both levels
 // hold the frame (no band fix-up).
-template <int IN_ = 4, int L1S_ = 5, int WIDE_ = 1>
+// BM: output tile rows (a multiple of 4).  BM = 28: 7 level-2 + 8 level-1 warps + the producer =
+// 16 warps, 4 per SM sub-partition with equal DMMA work on each (BM = 32: 18 warps, the
+// sub-partition holding warps 0, 4, 8, 12, 16 carries 138 DMMAs per plane against 108 on the
+// others), and the smaller planes leave room for a 5-deep input ring.
+// BAL (BM = 32 only): warp roles spread so the four SM sub-partitions (warp w runs on w mod 4)
+// carry equal DMMA work: sub-partition 0's five warps 0, 4, 8, 12, 16 and warps 1, 2, 3 are the
+// level-2 warps (24 DMMAs per plane each), warps 5-7, 9-11, 13-15 level 1 (30 each), warp 17
+// the producer: 120 / 114 / 114 / 114 DMMAs per plane instead of 138 / 108 / 108 / 108.
+template <int IN_ = 4, int L1S_ = 5, int WIDE_ = 1, int BM_ = 32, int BAL_ = 0>
 struct Tile3DTB2 {
+  static constexpr int BAL = BAL_;
   static constexpr int R = 1, A = 4, B = 2, KR = 6, KS = 6, H = 2, ZCH = 32;
   // WIDE = 1: 32 x 64 output tile, step-1 plane 36 x 80 (level-1 warps: 5 DMMA tiles each),
   //           inputs of output (row, col) at staged (row + dy, col + 1 + dx)   [OFF = 1]
@@ -1101,12 +1176,13 @@ struct Tile3DTB2 {
   //           inputs at staged (row + dy, col + dx)                             [OFF = 0]
   // (measured: WIDE = 1 312.7 GSt/s on Heat-3D, WIDE = 0 281 despite 9 % fewer DMMAs per output)
   static constexpr int WIDE = WIDE_, OFF = WIDE_;
-  static constexpr int BM = 32, BN = WIDE_ ? 64 : 62;   // output tile (stored)
+  static constexpr int BM = BM_, BN = WIDE_ ? 64 : 62;  // output tile (stored)
+  static_assert(BM % 4 == 0, "output tile rows");
   static constexpr int W1 = WIDE_ ? 5 : 4;               // level-1 DMMA tiles per warp
-  static constexpr int NL2 = 8, NL1 = 9;                 // level-2 / level-1 warps
+  static constexpr int NL2 = BM / 4, NL1 = BM / 4 + 1;   // level-2 / level-1 warps
   static constexpr int NT = 32 * (NL2 + NL1 + 1);
   static constexpr int TP = WIDE_ ? 84 : 68;             // plane pitch (input and step-1)
-  static constexpr int RIN = 38, R1 = 36;                // staged input rows, step-1 rows
+  static constexpr int RIN = BM + 6, R1 = BM + 4;        // staged input rows, step-1 rows
   static constexpr int SIN = RIN * TP, SIN_A = (SIN + 15) / 16 * 16;
   static constexpr int SL1 = R1 * TP, SL1_A = (SL1 + 15) / 16 * 16;
   // ring slots: input (3 read + IN - 3 in flight) and step-1 (3 read + 1 written + slack);
@@ -1135,7 +1211,7 @@ __device__ __forceinline__ void tb_hwindow(double (&acc)[G][2], const double* co
       for (int rho = 0; rho < C::KR; ++rho)
 #pragma unroll
         for (int j = 0; j < G; ++j) dmma_t(acc[j][0], acc[j][1], base[rho * C::TP + 16 * j], wf[ONE ? 0 : dz][rho]);
-    } else if (wz[dz] != 0.0) {
+    } else if (wz[dz] != 0.0) {  // (an integer mask test here measured 12 % slower: code layout)
 #pragma unroll
       for (int j = 0; j < G; ++j) {
         const double* v = pl[dz] + (r0 + alpha + C::R) * C::TP + c0 + 16 * j + C::B * g + beta + C::R + C::OFF;
@@ -1183,7 +1259,19 @@ __global__ void __launch_bounds__(D::NT, 1)
   __syncthreads();
   pdl_begin();
   const int ncol = a.tiles_x * a.tiles_y;
-  if (warp == D::NL2 + D::NL1) {  // producer: input planes z0-2 .. z1+1 of every item
+  // role: 0 level 2, 1 level 1, 2 producer; rb = the warp's row block within its level
+  int role, rb;
+  if constexpr (D::BAL) {
+    static_assert(!D::BAL || (D::NL2 == 8 && D::NL1 == 9), "balanced roles: 18 warps");
+    if (warp == 17) { role = 2; rb = 0; }
+    else if ((warp & 3) == 0) { role = 0; rb = warp >> 2; }     // 0, 4, 8, 12, 16 -> 0 .. 4
+    else if (warp < 4) { role = 0; rb = 4 + warp; }             // 1, 2, 3 -> 5, 6, 7
+    else { role = 1; rb = warp - 5 - (warp - 5) / 4; }         // 5-7, 9-11, 13-15 -> 0 .. 8
+  } else {
+    role = warp == D::NL2 + D::NL1 ? 2 : warp >= D::NL2 ? 1 : 0;
+    rb = role == 1 ? warp - D::NL2 : warp;
+  }
+  if (role == 2) {  // producer: input planes z0-2 .. z1+1 of every item
     if (lane == 0) tma_prefetch_desc(&tmap);
     int q = 0;
     for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
@@ -1214,9 +1302,9 @@ __global__ void __launch_bounds__(D::NT, 1)
   const int g = lane >> 2, t = lane & 3;
   const int alpha = (2 * t) / D::B, beta = (2 * t) % D::B;
   const bool fixed = a.hold_frame != 0;
-  if (warp >= D::NL2) {
+  if (role == 1) {
     // ---------------- level 1: step-1 planes ----------------
-    const int rb = warp - D::NL2;  // step-1 rows 4 rb .. 4 rb + 3, cols 0 .. 16 W1 - 1
+    // rb: step-1 rows 4 rb .. 4 rb + 3, cols 0 .. 16 W1 - 1
     int q = 0, p = 0;              // input / step-1 plane sequence numbers
     for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
       const int zcl = (int)(item / ncol), tile = (int)(item - (int64_t)zcl * ncol);
@@ -1272,7 +1360,7 @@ __global__ void __launch_bounds__(D::NT, 1)
     return;
   }
   // ---------------- level 2: output planes ----------------
-  const int rb = warp;  // output rows 4 rb .. 4 rb + 3, cols 0 .. 63 (BN stored)
+  // rb: output rows 4 rb .. 4 rb + 3, cols 0 .. 63 (BN stored)
   int p = 0;            // step-1 plane sequence number
   for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
     const int zcl = (int)(item / ncol), tile = (int)(item - (int64_t)zcl * ncol);
@@ -1356,6 +1444,9 @@ using Tile3D3c = Tile3DCfg<3, 8, 2, 4, 6, 32>;     // CTA 64 x 64 outputs, 8 DMM
 using Tile3D3d = Tile3DCfg<3, 2, 8, 1, 5, 32, 2>;  // CTA 64 x 32, 8 warps of 2 block rows x 2 column groups
 using Tile3D3k = Tile3DCfg<3, 8, 2, 2, 5, 32, 1, 1>;  // Tile3D3, k-slice-outer DMMA order
 using Tile3D3ck = Tile3DCfg<3, 8, 2, 4, 6, 32, 1, 1>;  // Tile3D3c, k-slice-outer DMMA order
+// Tile3D3 with the plane-interleaved row-outer order (KO = 2, box shapes only)
+using Tile3D3i = Tile3DCfg<3, 8, 2, 2, 5, 32, 1, 2>;
+using Tile3D3ci = Tile3DCfg<3, 8, 2, 4, 6, 32, 1, 2>;
 // wide tiles (the lateral x halo costs a 64-B DRAM granule on each side of every staged row:
 // 25 % extra reads at 64 columns, 12.5 % at 128; the TMA box is <= 256 wide): CTA 32 x 128
 // (8 warps of 2 column groups), 6-plane ring, 32- or 64-plane z chunks
@@ -1575,7 +1666,7 @@ static int tile1d_variant() {
 
 template <int NK>
 static cudaError_t launch_tile1d_nk(const S2RArgs& a, cudaStream_t st) {
-  if constexpr (NK == 15 || NK == 19 || NK == 21 || NK == 23) {  // tuning variants (CSX_TILE1D_VARIANT)
+  if constexpr (NK >= 15) {  // tuning variants (CSX_TILE1D_VARIANT)
     switch (tile1d_variant()) {
       case 1: return launch_tile1d_cfg<Tile1DCfg<NK, 512, 4, 4, 4>>(a, st);
       case 2: return launch_tile1d_cfg<Tile1DCfg<NK, 256, 4, 6, 2>>(a, st);
@@ -1690,7 +1781,15 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
       if (e && e[0] == '1') return launch_tile3d_tb<Tile3DTB>(a, a.tc_mask, st);
       const char* r = getenv("CSX_TB_GEOM");  // 0: the 32 x 62 tile (equal level work)
       if (r && r[0] == '0') return launch_tile3d_tb2<Tile3DTB2<5, 6, 0>>(a, a.tc_mask, st);
-      return launch_tile3d_tb2<Tile3DTB2<4, 5, 1>>(a, a.tc_mask, st);
+      if (r && r[0] == '3') return launch_tile3d_tb2<Tile3DTB2<5, 5, 1, 28>>(a, a.tc_mask, st);
+      if (r && r[0] == '4') return launch_tile3d_tb2<Tile3DTB2<4, 6, 1, 28>>(a, a.tc_mask, st);
+      if (r && r[0] == '5') return launch_tile3d_tb2<Tile3DTB2<6, 4, 1, 28>>(a, a.tc_mask, st);
+      if (r && r[0] == '6') return launch_tile3d_tb2<Tile3DTB2<5, 4, 1, 32>>(a, a.tc_mask, st);
+      // (BM = 28, geometries 3-5: 16 warps, balanced sub-partitions, deeper rings: 281-296 GSt/s, slower)
+      if (r && r[0] == '1') return launch_tile3d_tb2<Tile3DTB2<4, 5, 1>>(a, a.tc_mask, st);  // unbalanced roles
+      if (r && r[0] == '8') return launch_tile3d_tb2<Tile3DTB2<5, 4, 1, 32, 1>>(a, a.tc_mask, st);
+      // default: balanced roles (Heat-3D 315.0 -> 320.0 GSt/s)
+      return launch_tile3d_tb2<Tile3DTB2<4, 5, 1, 32, 1>>(a, a.tc_mask, st);
     }
     if (nk == 5 || nk == 7) {
       // k-slice-outer DMMA order by default (box r = 2 / 3: 56.4 -> 60.0 / 26.6 -> 27.6 GSt/s)
@@ -1728,6 +1827,10 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
       // (measured)
       // (k-slice-outer DMMA order: 287 vs 283 GSt/s on Heat-3D, but 184 vs 196 on Box-3D27P)
       if (__builtin_popcount((unsigned)a.tc_mask) <= 1) return launch_tile3d_cfg<Tile3D3ck>(a, a.tc_mask, st);
+      if (a.tc_mask == 7) {  // box: every plane on the tensor cores
+        if (e && e[0] == 'i') return launch_tile3d_cfg<Tile3D3i>(a, a.tc_mask, st);
+        if (e && e[0] == 'j') return launch_tile3d_cfg<Tile3D3ci>(a, a.tc_mask, st);
+      }
       return launch_tile3d_cfg<Tile3D3>(a, a.tc_mask, st);
     }
     return cudaErrorNotSupported;

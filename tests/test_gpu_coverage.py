@@ -299,3 +299,21 @@ def test_randomized_plans_against_oracle(csx):
         assert rel(got, ref) <= TOL, (case, ndim, r, box, tf, ext, bc, engine, T, cap)
         ran += 1
     assert ran >= 120, ran
+
+
+@pytest.mark.parametrize("geom", ["0", "1", "3", "4", "5", "6", "8"])
+def test_tb2_geometries(csx, monkeypatch, geom):
+    """Every k_tile3d_tb2 geometry (CSX_TB_GEOM; the default is the balanced-role 32 x 64 tile):
+    Heat-3D and Box-3D27P at Tf = 2, ragged tiles and z chunks, both boundaries, persistent grid
+    capped at 3 CTAs and uncapped, element-wise against the oracle."""
+    monkeypatch.setenv("CSX_TB_GEOM", geom)
+    for name, ext in (("heat3d", (70, 61, 150)), ("box3d27p", (40, 57, 130)), ("heat3d", (9, 29, 65))):
+        s = synth.SHAPES[name]
+        w = synth.random_weights(name)
+        u0 = synth.grid(ext, seed=5)
+        for bc in ("fixed", "periodic"):
+            ref = oracle.run(u0, w, bc, 5)
+            for cap in (3, 0):
+                got, info = run_gpu(csx, u0, w, s.kind, bc, 5, engine="tc_tile", fuse_steps=2, max_ctas=cap)
+                assert info["fuse_steps"] == 2
+                assert rel(got, ref) <= TOL, (geom, name, ext, bc, cap)
