@@ -1675,8 +1675,13 @@ static cudaError_t launch_tile1d_nk(const S2RArgs& a, cudaStream_t st) {
       case 5: return launch_tile1d_cfg<Tile1DCfg<NK, 128, 4, 8, 4>>(a, st);
       case 6: return launch_tile1d_cfg<Tile1DCfg<NK, 256, 8, 4, 4>>(a, st);
       case 7: return launch_tile1d_cfg<Tile1DCfg<NK, 256, 4, 6, 8>>(a, st);
+      case 8: return launch_tile1d_cfg<Tile1DCfg<NK, 256, 4, 6, 4>>(a, st);
     }
   }
+  // nk >= 21: 8 DMMA warps per CTA, 4-stage ring (variant 6; round-2 sweep: Heat-1D 102.4M at
+  // Tf = 13 3858 -> 4358 GSt/s, 10.24M 3263 -> 3727, 1D5P Tf = 7 2086 -> 2299); below that the
+  // 4-warp, 6-stage CTA (2 per SM) stays ahead (Tf = 7 / 9: 2435 / 3048 vs 2290 / 2941)
+  if constexpr (NK >= 21) return launch_tile1d_cfg<Tile1DCfg<NK, 256, 8, 4, 4>>(a, st);
   return launch_tile1d_cfg<Tile1DCfg<NK, 256, 4, 6, 4>>(a, st);  // 2 CTAs/SM x 4 DMMA warps
 }
 

@@ -676,3 +676,46 @@ def test_tile2d_variants(variant):
                          capture_output=True, text=True, timeout=300)
     assert out.returncode == 0, out.stderr[-2000:]
     assert float(out.stdout.strip().splitlines()[-1]) <= TOL, (variant, out.stdout)
+
+
+_TILE1D_SCRIPT = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+import oracle, synth
+import paper_conf_ppopp_chenlwbwmyzcy24_b200 as csx
+worst = 0.0
+for name, tf, T in (("heat1d", 7, 15), ("heat1d", 11, 23), ("heat1d", 13, 27), ("1d5p", 5, 11), ("1d5p", 7, 15)):
+    s = synth.SHAPES[name]
+    w = synth.random_weights(name)
+    u0 = synth.grid((70001,), seed=73)
+    for bc in ("fixed", "periodic"):
+        for cap in (3, 0):
+            p = csx.Plan(u0.shape, w, shape=s.kind, bc=bc, fuse_steps=tf, engine="tc_tile")
+            if cap:
+                p.set_max_ctas(cap)
+            d_in = torch.from_numpy(u0).cuda()
+            d_out = torch.empty_like(d_in)
+            p.run(d_in, d_out, T)
+            torch.cuda.synchronize()
+            ref = oracle.run(u0, w, bc, T)
+            worst = max(worst, float(np.max(np.abs(d_out.cpu().numpy() - ref)) / np.max(np.abs(ref))))
+            p.close()
+print(worst)
+"""
+
+
+@pytest.mark.parametrize("variant", ["1", "2", "3", "4", "5", "6", "7", "8"])
+def test_tile1d_variants(variant):
+    """Every 1D TC_TILE tile / warp / ring geometry (CSX_TILE1D_VARIANT, read once per process: a
+    subprocess each; the default — 8 DMMA warps for nk >= 21, variant 8's 4 warps below — runs in
+    the rest of the suite) at nk = 15, 23, 27 (r = 1) and 21, 29 (r = 2), with a remainder pass,
+    ragged tail, both boundaries, persistent grid capped at 3 CTAs and uncapped."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, "-c", _TILE1D_SCRIPT, root],
+                         env=dict(os.environ, CSX_TILE1D_VARIANT=variant), cwd=root,
+                         capture_output=True, text=True, timeout=300)
+    assert out.returncode == 0, out.stderr[-2000:]
+    assert float(out.stdout.strip().splitlines()[-1]) <= TOL, (variant, out.stdout)
