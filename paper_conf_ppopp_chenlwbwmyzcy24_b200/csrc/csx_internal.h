@@ -81,6 +81,9 @@ struct Padded {
   int64_t origin() const { return O[0] * s0 + O[1] * s1 + O[2]; }
 };
 
+// DMMAs per output point, pass and TC plane of the 3D Tf = 2 kernel that runs (kernels_tile.cu)
+double tile3d_tb_mma_per_point();
+
 }  // namespace csx
 
 // NVLink peer-memory halo exchange state of a sharded plan (comm.cpp, kernels_peer.cu).

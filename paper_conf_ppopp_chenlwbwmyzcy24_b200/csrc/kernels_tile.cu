@@ -18,6 +18,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <cstring>
 #include <cstdlib>
 
 #include "csx_run.h"
@@ -1438,6 +1439,295 @@ static cudaError_t launch_tile3d_tb2(S2RArgs a, int tc_mask, cudaStream_t st) {
   return launch_pdl(a.pdl != 0, kern, grid, D::NT, D::SMEM, st, a, tc_mask, tmap);
 }
 
+// ------------------------------------------------------------------------------------------
+// 3D Tf = 2, k_tile3d_tb3: k_tile3d_tb2's decoupled levels with the level-1 over-computation cut.
+// tb2's level 1 covers the 34 x 66 step-1 cells a 32 x 64 output tile needs with 45 DMMA tiles of
+// 4 x 16 (a 36 x 80 plane: 28 % of its DMMAs are wasted columns 67-79).  Here level 1 computes
+// step-1 columns 0-63 with 36 such tiles and columns 64-67 with 3 "strip" tiles whose 8 blocks
+// (4 x 2 each) sit one above the other (lane group g <-> row block g: every lane addresses its own
+// block, so a DMMA tile need not be a row of blocks): 39 tiles instead of 45, 420 DMMAs per plane
+// and TC plane instead of 462.  8 level-1 warps (tiles li, li + 8, ...: 5 / 5 / ... / 4), 8
+// level-2 warps and a producer = 17 warps, two level-1 and two level-2 warps per SM sub-partition
+// (DMMAs per plane 108 / 108 / 108 / 102 against tb2's best 120 / 114 / 114 / 114).  Input planes
+// are staged with a 76-column pitch (reads reach column 70; 2 x 76 = 24 banks mod 32 keeps the
+// single-tap plane loads conflict-free), step-1 planes with 68.
+// Measured (CSX_TB_GEOM a / b / c = ring depths 5+5 / 4+6 / 6+4): Heat-3D 294.5 / 301.4 / 281.0
+// GSt/s against tb2's 319.3 — 9 % fewer DMMAs and balanced sub-partitions do not pay: the
+// two-level pipeline is bound by its plane hand-offs, not by the DMMA pipe (52 % active) or the
+// smem wavefronts (~50 %).  Kept as a parity-tested variant, not the default.
+template <int IN_ = 5, int L1S_ = 5>
+struct Tile3DTB3 {
+  static constexpr int R = 1, A = 4, B = 2, KR = 6, KS = 6, H = 2, ZCH = 32;
+  static constexpr int BM = 32, BN = 64;
+  static constexpr int NL2 = 8, NL1 = 8, NTL1 = 39;  // warps per level, level-1 DMMA tiles
+  static constexpr int NT = 32 * (NL2 + NL1 + 1);
+  static constexpr int TPI = 76, TP1 = 68;          // input / step-1 plane pitch
+  static constexpr int C1 = 68;                     // step-1 columns computed (0 .. 67)
+  static constexpr int RIN = 38, R1 = 36;
+  static constexpr int SIN = RIN * TPI, SIN_A = (SIN + 15) / 16 * 16;
+  static constexpr int SL1 = R1 * TP1, SL1_A = (SL1 + 15) / 16 * 16;
+  static constexpr int IN = IN_, L1S = L1S_;
+  static constexpr int SMEM = (IN * SIN_A + L1S * SL1_A) * 8 + 128;
+  static_assert(SMEM <= 227 * 1024, "shared memory");
+};
+
+// block origin (row, col) of lane group g in level-1 tile tt (step-1 plane coordinates); `st`:
+// the lane group's block is a real one (tile 38 carries 2 blocks, its other groups repeat them)
+__device__ __forceinline__ void tb3_block(int tt, int g, int& row, int& col, bool& st) {
+  st = true;
+  if (tt < 36) {
+    row = 4 * (tt >> 2);
+    col = 16 * (tt & 3) + 2 * g;
+  } else if (tt < 38) {
+    row = 4 * g;
+    col = tt == 36 ? 64 : 66;
+  } else {
+    row = 32;
+    col = (g & 1) ? 66 : 64;
+    st = g < 2;
+  }
+}
+
+// G DMMA tiles, lane group g's block of tile j at staged-plane offset boff[j] (row * TPS + col):
+// the inputs of output (row, col) sit at (row + dy, col + 1 + dx) of the planes pl[dz] (pitch TPS)
+template <int G, int TPS, bool ONE>
+__device__ __forceinline__ void tb3_tiles(double (&acc)[G][2], const double* const (&pl)[3], const int (&boff)[G],
+                                          int tc_mask, const double (&wf)[ONE ? 1 : 3][6],
+                                          const double (&wz)[3], int t) {
+#pragma unroll
+  for (int j = 0; j < G; ++j) acc[j][0] = acc[j][1] = 0.0;
+#pragma unroll
+  for (int dz = 0; dz < 3; ++dz) {
+    if (tc_mask & (1 << dz)) {
+#pragma unroll
+      for (int rho = 0; rho < 6; ++rho)
+#pragma unroll
+        for (int j = 0; j < G; ++j)
+          dmma_t(acc[j][0], acc[j][1], pl[dz][boff[j] + rho * TPS + 1 + t], wf[ONE ? 0 : dz][rho]);
+    } else if (wz[dz] != 0.0) {
+#pragma unroll
+      for (int j = 0; j < G; ++j) {
+        const double2 v = *reinterpret_cast<const double2*>(pl[dz] + boff[j] + (t + 1) * TPS + 2);
+        acc[j][0] = fma(wz[dz], v.x, acc[j][0]);
+        acc[j][1] = fma(wz[dz], v.y, acc[j][1]);
+      }
+    }
+  }
+}
+
+// one level-1 step-1 plane for a warp's G tiles (tile li + 8 i): DMMA, FIXED frame, store
+template <int G, bool ONE, class D>
+__device__ __forceinline__ void tb3_level1(const double* const (&pin)[3], double* dl1, int li, int tc_mask,
+                                           const double (&wf)[ONE ? 1 : 3][6], const double (&wz)[3],
+                                           int g, int t, bool frame, bool zf1, int64_t sy0, int64_t sx0,
+                                           const S2RArgs& a) {
+  int boff[G];
+#pragma unroll
+  for (int i = 0; i < G; ++i) {
+    int r0, c0;
+    bool s0;
+    tb3_block(li + 8 * i, g, r0, c0, s0);
+    boff[i] = r0 * D::TPI + c0;
+  }
+  double acc[G][2];
+  tb3_tiles<G, D::TPI, ONE>(acc, pin, boff, tc_mask, wf, wz, t);
+#pragma unroll
+  for (int i = 0; i < G; ++i) {
+    int r0, c, s0;
+    bool st;
+    tb3_block(li + 8 * i, g, r0, c, st);
+    (void)s0;
+    const int r = r0 + t;  // this lane's two step-1 cells (r, c), (r, c + 1)
+    double v0 = acc[i][0], v1 = acc[i][1];
+    if (frame) {  // held frame points keep the input value
+      const int64_t gy = sy0 + r, gx = sx0 + c;
+      const double* ctr = pin[1] + (r + 1) * D::TPI + c + 2;
+      const bool yf = zf1 || gy < 1 || gy >= a.GE1 - 1;
+      if (yf || gx < 1 || gx >= a.GE2 - 1) v0 = ctr[0];
+      if (yf || gx + 1 < 1 || gx + 1 >= a.GE2 - 1) v1 = ctr[1];
+    }
+    if (st) *reinterpret_cast<double2*>(dl1 + r * D::TP1 + c) = make_double2(v0, v1);
+  }
+}
+
+template <bool ONE, class D>  // (17 warps: one SM sub-partition holds 5, so <= 96 registers)
+__global__ void __launch_bounds__(D::NT, 1)
+    k_tile3d_tb3(S2RArgs a, int tc_mask, const __grid_constant__ CUtensorMap tmap) {
+  extern __shared__ __align__(128) double smem_raw[];
+  double* smem = ring_base(smem_raw);
+  double* l1 = smem + D::IN * D::SIN_A;  // L1S step-1 planes
+  __shared__ __align__(8) uint64_t in_full[D::IN], in_empty[D::IN], l1_full[D::L1S], l1_empty[D::L1S];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  if (tid == 0) {
+    for (int s = 0; s < D::IN; ++s) {
+      mbar_init(&in_full[s], 1);
+      mbar_init(&in_empty[s], D::NL1);
+    }
+    for (int s = 0; s < D::L1S; ++s) {
+      mbar_init(&l1_full[s], D::NL1);
+      mbar_init(&l1_empty[s], D::NL2);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  __syncthreads();
+  pdl_begin();
+  const int ncol = a.tiles_x * a.tiles_y;
+  // warps 0-7 level 2 (output row block = warp), 8-15 level 1 (li = warp - 8), 16 producer
+  if (warp == D::NL2 + D::NL1) {  // producer: input planes z0-2 .. z1+1 of every item
+    if (lane == 0) tma_prefetch_desc(&tmap);
+    int q = 0;
+    for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
+      const int zcl = (int)(item / ncol), tile = (int)(item - (int64_t)zcl * ncol);
+      const int64_t zc = slab_map(a, zcl);
+      const int ty = tile / a.tiles_x, tx = tile - ty * a.tiles_x;
+      const int64_t z0 = zc * D::ZCH, z1 = min(a.E0, z0 + D::ZCH);
+      for (int64_t zi = z0 - D::H; zi < z1 + D::H; ++zi, ++q) {
+        const int s = q % D::IN, n = q / D::IN;
+        if (n > 0) mbar_wait(&in_empty[s], (uint32_t)((n - 1) & 1));
+        if (lane == 0) {
+          mbar_expect_tx(&in_full[s], (uint32_t)(D::SIN * 8));
+          tma_load_3d(smem + s * D::SIN_A, &tmap, &in_full[s], (int)(a.tma_x0 + (int64_t)tx * D::BN - 4),
+                      (int)(a.tma_y0 + (int64_t)ty * D::BM - 2), (int)(a.tma_z0 + zi));
+        }
+      }
+    }
+    return;
+  }
+  double wf[ONE ? 1 : 3][D::KS], wz[3];
+  const int dz1 = __ffs(tc_mask) - 1;
+#pragma unroll
+  for (int p = 0; p < (ONE ? 1 : 3); ++p)
+#pragma unroll
+    for (int k = 0; k < D::KS; ++k) wf[p][k] = a.frags[((ONE ? dz1 : p) * D::KS + k) * 32 + lane];
+#pragma unroll
+  for (int p = 0; p < 3; ++p) wz[p] = a.wc[(p * 3 + 1) * 3 + 1];
+  const int g = lane >> 2, t = lane & 3;
+  const bool fixed = a.hold_frame != 0;
+  if (warp >= D::NL2) {
+    // ---------------- level 1: step-1 planes (cols 0 .. 67; col c <-> x0 - 2 + c) ----------------
+    const int li = warp - D::NL2;
+    int q = 0, p = 0;  // input / step-1 plane sequence numbers
+    for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
+      const int zcl = (int)(item / ncol), tile = (int)(item - (int64_t)zcl * ncol);
+      const int64_t zc = slab_map(a, zcl);
+      const int ty = tile / a.tiles_x, tx = tile - ty * a.tiles_x;
+      const int64_t z0 = zc * D::ZCH, z1 = min(a.E0, z0 + D::ZCH);
+      const int64_t sy0 = (int64_t)ty * D::BM + a.gorg1 - 1, sx0 = (int64_t)tx * D::BN + a.gorg2 - 2;
+      const bool tile_edge = fixed && (sy0 < 1 || sy0 + D::R1 > a.GE1 - 1 || sx0 < 1 || sx0 + D::C1 > a.GE2 - 1);
+      const int q0 = q;  // input plane z0-2 of this item
+      auto in_slot = [&](int qq) { return smem + (qq % D::IN) * D::SIN_A; };
+      mbar_wait(&in_full[q0 % D::IN], (uint32_t)((q0 / D::IN) & 1));
+      mbar_wait(&in_full[(q0 + 1) % D::IN], (uint32_t)(((q0 + 1) / D::IN) & 1));
+      for (int64_t k = z0 - 1; k <= z1; ++k, ++p) {
+        const int j = (int)(k - (z0 - 1));
+        mbar_wait(&in_full[(q0 + j + 2) % D::IN], (uint32_t)(((q0 + j + 2) / D::IN) & 1));
+        const int sl = p % D::L1S, nl = p / D::L1S;
+        if (nl > 0) mbar_wait(&l1_empty[sl], (uint32_t)((nl - 1) & 1));
+        const double* pin[3] = {in_slot(q0 + j), in_slot(q0 + j + 1), in_slot(q0 + j + 2)};
+        double* dl1 = l1 + sl * D::SL1_A;
+        const int64_t gz1 = k + a.gorg0;
+        const bool zf1 = fixed && (gz1 < 1 || gz1 >= a.GE0 - 1);
+        const bool frame = fixed && (zf1 || tile_edge);
+        if (li + 32 < D::NTL1)
+          tb3_level1<5, ONE, D>(pin, dl1, li, tc_mask, wf, wz, g, t, frame, zf1, sy0, sx0, a);
+        else
+          tb3_level1<4, ONE, D>(pin, dl1, li, tc_mask, wf, wz, g, t, frame, zf1, sy0, sx0, a);
+        __syncwarp();
+        if (lane == 0) {
+          mbar_arrive(&l1_full[sl]);                 // this warp's cells of plane k written
+          mbar_arrive(&in_empty[(q0 + j) % D::IN]);  // input plane k-1 no longer read
+        }
+      }
+      __syncwarp();
+      if (lane == 0) {  // input planes z1, z1+1 (read by the last step-1 plane only)
+        mbar_arrive(&in_empty[(q0 + (int)(z1 - z0) + 2) % D::IN]);
+        mbar_arrive(&in_empty[(q0 + (int)(z1 - z0) + 3) % D::IN]);
+      }
+      q = q0 + (int)(z1 - z0) + 4;
+    }
+    return;
+  }
+  // ---------------- level 2: output planes ----------------
+  const int rb = warp;  // output rows 4 rb .. 4 rb + 3, cols 0 .. 63
+  int boff[4];
+#pragma unroll
+  for (int jj = 0; jj < 4; ++jj) boff[jj] = 4 * rb * D::TP1 + 16 * jj + 2 * g;
+  int p = 0;  // step-1 plane sequence number
+  for (int64_t item = blockIdx.x; item < a.ntiles; item += gridDim.x) {
+    const int zcl = (int)(item / ncol), tile = (int)(item - (int64_t)zcl * ncol);
+    const int64_t zc = slab_map(a, zcl);
+    const int ty = tile / a.tiles_x, tx = tile - ty * a.tiles_x;
+    const int64_t z0 = zc * D::ZCH, z1 = min(a.E0, z0 + D::ZCH);
+    const int64_t y0 = (int64_t)ty * D::BM, x0 = (int64_t)tx * D::BN;
+    const int64_t gy0 = y0 + a.gorg1, gx0 = x0 + a.gorg2;
+    const bool tile_edge = fixed && (gy0 < 1 || gy0 + D::BM > a.GE1 - 1 || gx0 < 1 || gx0 + D::BN > a.GE2 - 1);
+    const int p0 = p;  // step-1 plane z0-1 of this item
+    auto l1_slot = [&](int pp) { return l1 + (pp % D::L1S) * D::SL1_A; };
+    auto l1_wait = [&](int pp) { mbar_wait(&l1_full[pp % D::L1S], (uint32_t)((pp / D::L1S) & 1)); };
+    l1_wait(p0);
+    l1_wait(p0 + 1);
+    for (int64_t zo = z0; zo < z1; ++zo) {
+      const int j = (int)(zo - z0);
+      l1_wait(p0 + j + 2);
+      const double* p1[3] = {l1_slot(p0 + j), l1_slot(p0 + j + 1), l1_slot(p0 + j + 2)};
+      double acc[4][2];
+      tb3_tiles<4, D::TP1, ONE>(acc, p1, boff, tc_mask, wf, wz, t);
+      const int64_t gzo = zo + a.gorg0;
+      const bool zf = fixed && (gzo < 1 || gzo >= a.GE0 - 1);
+      double* plane = a.dst.p + zo * a.dst.s0;
+#pragma unroll
+      for (int jj = 0; jj < 4; ++jj) {
+        const int r = 4 * rb + t, c = 16 * jj + 2 * g;  // output tile coords
+        const int64_t row = y0 + r, col = x0 + c;
+        double v0 = acc[jj][0], v1 = acc[jj][1];
+        if (fixed && (zf || tile_edge)) {
+          const double* ctr = p1[1] + (r + 1) * D::TP1 + c + 2;
+          const int64_t gy = gy0 + r, gx = gx0 + c;
+          const bool yf = zf || gy < 1 || gy >= a.GE1 - 1;
+          if (yf || gx < 1 || gx >= a.GE2 - 1) v0 = ctr[0];
+          if (yf || gx + 1 < 1 || gx + 1 >= a.GE2 - 1) v1 = ctr[1];
+        }
+        if (row >= a.E1 || col >= a.E2) continue;
+        double* pp = plane + row * a.dst.s1 + col;
+        if (col + 1 < a.E2 && a.dst_aligned) {
+          *reinterpret_cast<double2*>(pp) = make_double2(v0, v1);
+        } else {
+          pp[0] = v0;
+          if (col + 1 < a.E2) pp[1] = v1;
+        }
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&l1_empty[(p0 + j) % D::L1S]);  // step-1 plane zo-1 done
+    }
+    __syncwarp();
+    if (lane == 0) {  // step-1 planes z1-1, z1 (read by the last output plane only)
+      mbar_arrive(&l1_empty[(p0 + (int)(z1 - z0)) % D::L1S]);
+      mbar_arrive(&l1_empty[(p0 + (int)(z1 - z0) + 1) % D::L1S]);
+    }
+    p = p0 + (int)(z1 - z0) + 2;
+  }
+}
+
+template <class D>
+static cudaError_t launch_tile3d_tb3(S2RArgs a, int tc_mask, cudaStream_t st) {
+  a.dst_aligned = ((reinterpret_cast<uintptr_t>(a.dst.p) & 15) == 0) && (a.dst.s1 % 2 == 0) &&
+                  (a.dst.s0 % 2 == 0);
+  a.tiles_x = (int)((a.E2 + D::BN - 1) / D::BN);
+  a.tiles_y = (int)((a.E1 + D::BM - 1) / D::BM);
+  a.ntiles = (int64_t)a.tiles_x * a.tiles_y * set_ranges(a, (a.E0 + D::ZCH - 1) / D::ZCH, D::ZCH, a.E0, D::H);
+  if (a.ntiles == 0) return cudaSuccess;
+  CUtensorMap tmap;
+  if (!make_tmap(a, D::TPI, D::RIN, &tmap)) return cudaErrorNotSupported;
+  auto kern = __builtin_popcount((unsigned)tc_mask) == 1 ? k_tile3d_tb3<true, D> : k_tile3d_tb3<false, D>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, D::SMEM);
+  if (e != cudaSuccess) return e;
+  int occ = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, D::NT, D::SMEM);
+  if (e != cudaSuccess) return e;
+  const int64_t grid = persistent_grid(occ, a.max_ctas, a.ntiles);
+  return launch_pdl(a.pdl != 0, kern, grid, D::NT, D::SMEM, st, a, tc_mask, tmap);
+}
+
 using Tile3D3 = Tile3DCfg<3, 8, 2, 2, 5, 32>;      // CTA 64 x 32 outputs, 4 DMMA warps, 5-plane ring, 32 planes per item
 using Tile3D3b = Tile3DCfg<3, 4, 4, 1, 5, 32, 2>;  // CTA 64 x 32, 4 warps of 4 block rows x 2 column groups
 using Tile3D3c = Tile3DCfg<3, 8, 2, 4, 6, 32>;     // CTA 64 x 64 outputs, 8 DMMA warps, 6-plane ring
@@ -1706,6 +1996,28 @@ static cudaError_t launch_tile1d(int nk, const S2RArgs& a, cudaStream_t st) {
   return cudaErrorNotSupported;
 }
 
+// 3D Tf = 2 geometry (CSX_TB_GEOM, read per call; the planner's DMMA count follows the same
+// choice): '0' tb2 32 x 62, '1' tb2 32 x 64 roles by warp index, 't' tb2 32 x 64 balanced roles,
+// '3'-'5' tb2 28 x 64, '6' / '8' tb2 ring depths, 'a'-'c' tb3 strip tiles
+#define CSX_TB_GEOM_DEFAULT 't'
+static char tb_geom() {
+  const char* r = getenv("CSX_TB_GEOM");
+  if (r && r[0] && std::strchr("0134568abct", r[0])) return r[0];
+  return CSX_TB_GEOM_DEFAULT;  // balanced roles (Heat-3D 315.0 -> 320.0 GSt/s)
+}
+
+// DMMAs per output point and pass, per TC plane of the base window, of the Tf = 2 geometry that
+// runs: (level-1 DMMA tiles x 34 / 32 planes — the z chunk's two extra step-1 planes — + level-2
+// tiles) x 6 DMMAs (K = 24) per tile, over the output tile's points
+double tile3d_tb_mma_per_point() {
+  switch (tb_geom()) {
+    case '0': return (36.0 * 34.0 / 32.0 + 32.0) * 6.0 / (32.0 * 62.0);  // step-1 36 x 64
+    case '3': case '4': case '5': return (40.0 * 34.0 / 32.0 + 28.0) * 6.0 / (28.0 * 64.0);
+    case 'a': case 'b': case 'c': return (39.0 * 34.0 / 32.0 + 32.0) * 6.0 / (32.0 * 64.0);
+    default: return (45.0 * 34.0 / 32.0 + 32.0) * 6.0 / (32.0 * 64.0);  // step-1 36 x 80
+  }
+}
+
 // (ndim, base radius, fused steps) -> is there a TC_TILE kernel for the pass?  3D: Tf = 1 runs
 // the per-plane GEMM of the composed window (= the base window) for r = 1..3 (nk = 3, 5, 7);
 // Tf = 2 only by the temporal blocking of the base r = 1 stencil (k_tile3d_tb).
@@ -1784,7 +2096,8 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
     if (tf == 2) {  // r = 1: temporal blocking (CSX_TB=1: the round-1 single-barrier kernel)
       const char* e = getenv("CSX_TB");
       if (e && e[0] == '1') return launch_tile3d_tb<Tile3DTB>(a, a.tc_mask, st);
-      const char* r = getenv("CSX_TB_GEOM");  // 0: the 32 x 62 tile (equal level work)
+      const char g = tb_geom();
+      const char* r = &g;  // 0: the 32 x 62 tile (equal level work)
       if (r && r[0] == '0') return launch_tile3d_tb2<Tile3DTB2<5, 6, 0>>(a, a.tc_mask, st);
       if (r && r[0] == '3') return launch_tile3d_tb2<Tile3DTB2<5, 5, 1, 28>>(a, a.tc_mask, st);
       if (r && r[0] == '4') return launch_tile3d_tb2<Tile3DTB2<4, 6, 1, 28>>(a, a.tc_mask, st);
@@ -1792,9 +2105,12 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
       if (r && r[0] == '6') return launch_tile3d_tb2<Tile3DTB2<5, 4, 1, 32>>(a, a.tc_mask, st);
       // (BM = 28, geometries 3-5: 16 warps, balanced sub-partitions, deeper rings: 281-296 GSt/s, slower)
       if (r && r[0] == '1') return launch_tile3d_tb2<Tile3DTB2<4, 5, 1>>(a, a.tc_mask, st);  // unbalanced roles
+      if (r && r[0] == 't') return launch_tile3d_tb2<Tile3DTB2<4, 5, 1, 32, 1>>(a, a.tc_mask, st);
+      if (r && r[0] == 'a') return launch_tile3d_tb3<Tile3DTB3<5, 5>>(a, a.tc_mask, st);
+      if (r && r[0] == 'b') return launch_tile3d_tb3<Tile3DTB3<4, 6>>(a, a.tc_mask, st);
+      if (r && r[0] == 'c') return launch_tile3d_tb3<Tile3DTB3<6, 4>>(a, a.tc_mask, st);
       if (r && r[0] == '8') return launch_tile3d_tb2<Tile3DTB2<5, 4, 1, 32, 1>>(a, a.tc_mask, st);
-      // default: balanced roles (Heat-3D 315.0 -> 320.0 GSt/s)
-      return launch_tile3d_tb2<Tile3DTB2<4, 5, 1, 32, 1>>(a, a.tc_mask, st);
+      return cudaErrorNotSupported;
     }
     if (nk == 5 || nk == 7) {
       // k-slice-outer DMMA order by default (box r = 2 / 3: 56.4 -> 60.0 / 26.6 -> 27.6 GSt/s)

@@ -312,14 +312,15 @@ csx_status build_pass(const csx_plan_s* p, int tf, Pass* out) {
     // 3D Tf = 2 runs the BASE stencil twice by temporal blocking (k_tile3d_tb2), not the composed
     // window: per 32 x 64 output tile and plane, level 1 computes 45 DMMA tiles (4 x 16) on the
     // grown 36 x 80 tile for 34 of every 32 planes (the z-chunk's two extra step-1 planes) and
-    // level 2 32 tiles, 6 DMMAs (K = 24) per tile and TC plane of the base window.
+    // level 2 32 tiles, 6 DMMAs (K = 24) per tile and TC plane of the base window (k_tile3d_tb3:
+    // 39 level-1 tiles; tile3d_tb_mma_per_point follows the geometry the launch will pick).
     int base_tc = 0;
     for (int dz = 0; dz < 3; ++dz) {
       int taps = 0;
       for (int i = 0; i < 9; ++i) taps += p->w[(size_t)dz * 9 + i] != 0.0;
       base_tc += taps > 1;
     }
-    P.tile_mma_per_pass = (int64_t)((double)pts / 2048.0 * (45.0 * 34.0 / 32.0 + 32.0) * 6 * base_tc + 0.5);
+    P.tile_mma_per_pass = (int64_t)((double)pts * tile3d_tb_mma_per_point() * base_tc + 0.5);
   }
   *out = std::move(P);
   return CSX_OK;

@@ -301,9 +301,10 @@ def test_randomized_plans_against_oracle(csx):
     assert ran >= 120, ran
 
 
-@pytest.mark.parametrize("geom", ["0", "1", "3", "4", "5", "6", "8"])
+@pytest.mark.parametrize("geom", ["0", "1", "3", "4", "5", "6", "8", "a", "b", "c", "t"])
 def test_tb2_geometries(csx, monkeypatch, geom):
-    """Every k_tile3d_tb2 geometry (CSX_TB_GEOM; the default is the balanced-role 32 x 64 tile):
+    """Every k_tile3d_tb2 / k_tile3d_tb3 geometry (CSX_TB_GEOM; a-c: tb3's strip tiles with three
+    ring depths, t: the balanced-role tb2 32 x 64 tile):
     Heat-3D and Box-3D27P at Tf = 2, ragged tiles and z chunks, both boundaries, persistent grid
     capped at 3 CTAs and uncapped, element-wise against the oracle."""
     monkeypatch.setenv("CSX_TB_GEOM", geom)

@@ -333,3 +333,26 @@ def test_run_argument_validation_without_gpu():
 def test_status_strings():
     for code in range(7):
         assert csx._lib.csx_status_string(code).decode().startswith("CSX_")
+
+
+@pytest.mark.parametrize("geom, l1_tiles, rows, cols", [
+    (None, 45, 32, 64), ("t", 45, 32, 64), ("1", 45, 32, 64), ("a", 39, 32, 64), ("c", 39, 32, 64),
+    ("3", 40, 28, 64), ("0", 36, 32, 62)])
+def test_3d_two_step_mma_count(monkeypatch, geom, l1_tiles, rows, cols):
+    """3D Tf = 2 (temporal blocking of the base r = 1 window): the planner's DMMA count per pass
+    follows the geometry CSX_TB_GEOM selects — (level-1 DMMA tiles x 34/32 planes + level-2
+    tiles) x 6 DMMAs per tile and TC plane, over the output tile's points: 1 TC plane for
+    Heat-3D, 3 for Box-3D27P."""
+    if geom is None:
+        monkeypatch.delenv("CSX_TB_GEOM", raising=False)
+    else:
+        monkeypatch.setenv("CSX_TB_GEOM", geom)
+    ext = (64, 96, 128)
+    pts = ext[0] * ext[1] * ext[2]
+    l2_tiles = rows // 4 * 4
+    per_pt = (l1_tiles * 34 / 32 + l2_tiles) * 6 / (rows * cols)
+    for name, ntc in (("heat3d", 1), ("box3d27p", 3)):
+        s = synth.SHAPES[name]
+        p = csx.Plan(ext, synth.physical_weights(name), shape=s.kind, fuse_steps=2)
+        assert p.info()["mma_per_pass"] == int(pts * per_pt * ntc + 0.5), (geom, name)
+        p.close()
