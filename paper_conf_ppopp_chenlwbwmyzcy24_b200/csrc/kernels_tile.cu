@@ -1764,6 +1764,12 @@ using Tile3D5g = Tile3DCfg<5, 8, 4, 2, 6, 32, 1, 1, 2, 4, 0>;
 // mod 32: the four block rows of one 8-lane LDS.128 phase fall on disjoint banks)
 using Tile3D5gc = Tile3DCfg<5, 8, 4, 2, 6, 32, 1, 1, 2, 4, 0, 0, 1>;
 using Tile3D7ks = Tile3DCfg<7, 4, 2, 4, 10, 32, 1, 1, 4, 2, 0, 4>;
+// 16 DMMA warps per CTA (CSX_TILE3D_W16; the 8-warp star kernels keep the DMMA pipe ~50 % busy):
+// default for r = 2 stars (+4.6 %); r = 3 stars (spills at 96 registers) and Heat-3D (271 vs 295)
+// measured slower
+using Tile3D5w = Tile3DCfg<5, 4, 8, 2, 6, 32, 1, 1, 2, 4, 0, 0, 1>;
+using Tile3D7w = Tile3DCfg<7, 2, 4, 4, 10, 32, 1, 1, 4, 2, 0, 4>;
+using Tile3D3w16 = Tile3DCfg<3, 4, 4, 4, 6, 32, 1, 1>;
 
 
 // ------------------------------------------------------------------------------------------
@@ -2123,6 +2129,12 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
       // star: conflict-free DFMA plane loads (CSX_STAR_CF = 0: the round-2 layouts)
       const char* cf = getenv("CSX_STAR_CF");
       const bool scf = star && !(cf && cf[0] == '0');
+      // 16 DMMA warps (CSX_TILE3D_W16): the default for r = 2 stars (Star-3D13P 190.5 -> 199.2
+      // GSt/s); r = 3 stars spill at 16 warps (121.7 -> 96.4) and keep 8 unless W16 = 1
+      const char* w16 = getenv("CSX_TILE3D_W16");
+      const bool w16_on = w16 ? w16[0] == '1' : nk == 5;
+      if (star && scf && w16_on)
+        return nk == 5 ? launch_tile3d_cfg<Tile3D5w>(a, a.tc_mask, st) : launch_tile3d_cfg<Tile3D7w>(a, a.tc_mask, st);
       if (nk == 5 && (g8 ? g8[0] == '1' : star))
         return scf ? launch_tile3d_cfg<Tile3D5gc>(a, a.tc_mask, st) : launch_tile3d_cfg<Tile3D5g>(a, a.tc_mask, st);
       if (nk == 7 && scf && ko) return launch_tile3d_cfg<Tile3D7ks>(a, a.tc_mask, st);
@@ -2147,7 +2159,11 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
       // (less halo per plane); box shapes (DMMA-bound) the 64 x 32 tile at 2 CTAs / SM
       // (measured)
       // (k-slice-outer DMMA order: 287 vs 283 GSt/s on Heat-3D, but 184 vs 196 on Box-3D27P)
-      if (__builtin_popcount((unsigned)a.tc_mask) <= 1) return launch_tile3d_cfg<Tile3D3ck>(a, a.tc_mask, st);
+      if (__builtin_popcount((unsigned)a.tc_mask) <= 1) {
+        const char* w16 = getenv("CSX_TILE3D_W16");
+        if (w16 && w16[0] == '1') return launch_tile3d_cfg<Tile3D3w16>(a, a.tc_mask, st);
+        return launch_tile3d_cfg<Tile3D3ck>(a, a.tc_mask, st);
+      }
       if (a.tc_mask == 7) {  // box: every plane on the tensor cores
         if (e && e[0] == 'i') return launch_tile3d_cfg<Tile3D3i>(a, a.tc_mask, st);
         if (e && e[0] == 'j') return launch_tile3d_cfg<Tile3D3ci>(a, a.tc_mask, st);

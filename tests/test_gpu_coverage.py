@@ -240,7 +240,7 @@ def test_graph_plan_variant_switch_teardown(csx):
 
 
 @pytest.mark.parametrize("env", [{"CSX_TILE3D_KO": "0"}, {"CSX_TILE3D5_G8": "1"}, {"CSX_TILE3D5_G8": "0"},
-                                 {"CSX_STAR_CF": "0"}])
+                                 {"CSX_STAR_CF": "0"}, {"CSX_TILE3D_W16": "0"}, {"CSX_TILE3D_W16": "1"}])
 def test_parity_3d_general_radius_variants(csx, monkeypatch, env):
     """The other 3D r = 2 / 3 tile configurations (row-outer DMMA order; 8 or 4 blocks per warp
     for both stars and boxes; the round-2 star layouts without the conflict-free DFMA planes;
@@ -318,3 +318,17 @@ def test_tb2_geometries(csx, monkeypatch, geom):
                 got, info = run_gpu(csx, u0, w, s.kind, bc, 5, engine="tc_tile", fuse_steps=2, max_ctas=cap)
                 assert info["fuse_steps"] == 2
                 assert rel(got, ref) <= TOL, (geom, name, ext, bc, cap)
+
+
+def test_heat3d_tf1_16_warps(csx, monkeypatch):
+    """The 16-DMMA-warp Heat-3D Tf = 1 tile (CSX_TILE3D_W16 = 1, an A/B variant): ragged tiles,
+    z chunks, both boundaries, capped and uncapped persistent grids."""
+    monkeypatch.setenv("CSX_TILE3D_W16", "1")
+    s = synth.SHAPES["heat3d"]
+    w = synth.random_weights("heat3d")
+    u0 = synth.grid((45, 70, 130), seed=11)
+    for bc in ("fixed", "periodic"):
+        ref = oracle.run(u0, w, bc, 3)
+        for cap in (3, 0):
+            got, _ = run_gpu(csx, u0, w, s.kind, bc, 3, engine="tc_tile", fuse_steps=1, max_ctas=cap)
+            assert rel(got, ref) <= TOL, (bc, cap)
