@@ -535,8 +535,10 @@ static int tile_variant() {
 // adjacent and the DFMA planes load them as two conflict-free LDS.64 rows instead of one
 // 2-way-conflicted LDS.128 (round 2: 36 M smem load conflicts per Star-3D13P launch).
 template <int NK_, int G_, int WM_, int WN_, int STAGES_, int ZCH_, int CG_ = 1, int KO_ = 0,
-          int A_ = 4, int B_ = 2, int WREG_ = 1, int TPX_ = 0, int CM_ = 0>
+          int A_ = 4, int B_ = 2, int WREG_ = 1, int TPX_ = 0, int CM_ = 0, int MINB_ = 0>
 struct Tile3DCfg {
+  // resident CTAs per SM the register budget is sized for (0: 1 above 4 DMMA warps, else 2)
+  static constexpr int MINB = MINB_ ? MINB_ : (WM_ * WN_ > 4 ? 1 : 2);
   static constexpr int NK = NK_, A = A_, B = B_, KC = 4 * ((B_ + NK - 1 + 3) / 4), G = G_, WM = WM_,
                        WN = WN_, STAGES = STAGES_, ZCH = ZCH_, CG = CG_;
   static constexpr int WREG = WREG_;  // 1: all planes' weight fragments live in registers
@@ -584,7 +586,7 @@ __device__ __forceinline__ void issue_plane(const S2RArgs& a, const CUtensorMap*
 __device__ __forceinline__ int ring_next(int s, int n) { return s + 1 == n ? 0 : s + 1; }
 
 template <class C, bool ONE = false>  // ONE: a single TC plane (star shapes)
-__global__ void __launch_bounds__(C::NT, (C::NCW > 4 ? 1 : 2))
+__global__ void __launch_bounds__(C::NT, C::MINB)
     k_tile3d(S2RArgs a, int tc_mask, const __grid_constant__ CUtensorMap tmap) {
   extern __shared__ __align__(128) double smem_raw[];
   double* smem = ring_base(smem_raw);
@@ -1770,6 +1772,12 @@ using Tile3D7ks = Tile3DCfg<7, 4, 2, 4, 10, 32, 1, 1, 4, 2, 0, 4>;
 using Tile3D5w = Tile3DCfg<5, 4, 8, 2, 6, 32, 1, 1, 2, 4, 0, 0, 1>;
 using Tile3D7w = Tile3DCfg<7, 2, 4, 4, 10, 32, 1, 1, 4, 2, 0, 4>;
 using Tile3D3w16 = Tile3DCfg<3, 4, 4, 4, 6, 32, 1, 1>;
+using Tile3D3w16r = Tile3DCfg<3, 4, 4, 4, 6, 32, 1, 0>;  // row-outer DMMA order (boxes)
+using Tile3D5w16 = Tile3DCfg<5, 2, 8, 2, 9, 32, 1, 1, 2, 4, 0>;  // box r = 2, 16 warps, CTA 32 x 64
+using Tile3D7w16 = Tile3DCfg<7, 2, 4, 4, 10, 32, 1, 1, 4, 2, 0>;  // box r = 3, 16 warps, CTA 32 x 64
+// box r = 1: two CTAs of 8 DMMA warps per SM (CTA 64 x 32), row-outer / k-slice-outer order
+using Tile3D3m2 = Tile3DCfg<3, 4, 4, 2, 5, 32, 1, 0, 4, 2, 1, 0, 0, 2>;
+using Tile3D3m2k = Tile3DCfg<3, 4, 4, 2, 5, 32, 1, 1, 4, 2, 1, 0, 0, 2>;
 
 
 // ------------------------------------------------------------------------------------------
@@ -2138,6 +2146,10 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
       if (nk == 5 && (g8 ? g8[0] == '1' : star))
         return scf ? launch_tile3d_cfg<Tile3D5gc>(a, a.tc_mask, st) : launch_tile3d_cfg<Tile3D5g>(a, a.tc_mask, st);
       if (nk == 7 && scf && ko) return launch_tile3d_cfg<Tile3D7ks>(a, a.tc_mask, st);
+      // boxes: 16 DMMA warps for r = 2 / 3 by default (Box-3D125P 59.8 -> 70.7 GSt/s, 0.78 ->
+      // 0.92 of the DMMA roof; Box-3D343P 27.5 -> 31.3, 0.83 -> 0.95); CSX_TILE3D_W16 = 0: 8 warps
+      if (nk == 5 && !star && !(w16 && w16[0] == '0')) return launch_tile3d_cfg<Tile3D5w16>(a, a.tc_mask, st);
+      if (nk == 7 && !star && !(w16 && w16[0] == '0')) return launch_tile3d_cfg<Tile3D7w16>(a, a.tc_mask, st);
       if (nk == 5) return ko ? launch_tile3d_cfg<Tile3D5k>(a, a.tc_mask, st) : launch_tile3d_cfg<Tile3D5>(a, a.tc_mask, st);
       return ko ? launch_tile3d_cfg<Tile3D7k>(a, a.tc_mask, st) : launch_tile3d_cfg<Tile3D7>(a, a.tc_mask, st);
     }
@@ -2165,6 +2177,10 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
         return launch_tile3d_cfg<Tile3D3ck>(a, a.tc_mask, st);
       }
       if (a.tc_mask == 7) {  // box: every plane on the tensor cores
+        if (e && e[0] == 'w') return launch_tile3d_cfg<Tile3D3w16>(a, a.tc_mask, st);
+        if (e && e[0] == 'x') return launch_tile3d_cfg<Tile3D3w16r>(a, a.tc_mask, st);
+        if (e && e[0] == 'm') return launch_tile3d_cfg<Tile3D3m2>(a, a.tc_mask, st);
+        if (e && e[0] == 'n') return launch_tile3d_cfg<Tile3D3m2k>(a, a.tc_mask, st);
         if (e && e[0] == 'i') return launch_tile3d_cfg<Tile3D3i>(a, a.tc_mask, st);
         if (e && e[0] == 'j') return launch_tile3d_cfg<Tile3D3ci>(a, a.tc_mask, st);
       }

@@ -1,0 +1,28 @@
+#!/bin/bash
+OUT=gpurun_out/r02b16c; mkdir -p $OUT
+B="python bench.py --steps 5 --warmup 3 --no-cpu-baseline --no-e2e --no-comparator"
+for v in 0 m n; do echo "box3d27p v=$v $(CSX_TILE3D_VARIANT=$v timeout 300 $B --config box3d27p_512 2>/dev/null)" >> $OUT/ab.txt; done
+echo "box3d343p default $(timeout 600 python bench.py --steps 3 --warmup 3 --no-cpu-baseline --no-e2e --no-comparator --config box3d343p_512 2>/dev/null)" >> $OUT/ab.txt
+cat > /tmp/b16c.py <<'PY'
+import os, sys, numpy as np, torch
+sys.path.insert(0, ".")
+import oracle, synth
+import paper_conf_ppopp_chenlwbwmyzcy24_b200 as csx
+worst = 0.0
+for v in ("m", "n"):
+    os.environ["CSX_TILE3D_VARIANT"] = v
+    s = synth.SHAPES["box3d27p"]; w = synth.random_weights("box3d27p")
+    for ext in ((45, 37, 70), (40, 70, 130)):
+        u0 = synth.grid(ext, seed=9)
+        for bc in ("fixed", "periodic"):
+            for cap in (3, 0):
+                p = csx.Plan(ext, w, shape=s.kind, bc=bc, fuse_steps=1, engine="tc_tile")
+                if cap: p.set_max_ctas(cap)
+                d_in = torch.from_numpy(u0).cuda(); d_out = torch.empty_like(d_in)
+                p.run(d_in, d_out, 3); torch.cuda.synchronize()
+                ref = oracle.run(u0, w, bc, 3)
+                e = float(np.max(np.abs(d_out.cpu().numpy() - ref)) / np.max(np.abs(ref))); p.close()
+                worst = max(worst, e); assert e <= 1e-12, (v, ext, bc, cap, e)
+print("box16c worst rel err", worst)
+PY
+timeout 300 python /tmp/b16c.py > $OUT/parity.txt 2>&1

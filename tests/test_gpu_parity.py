@@ -286,10 +286,12 @@ def test_parity_3d_two_step_blocking(csx, name, bc):
         del os.environ["CSX_FORCE_OVERLAP"]
 
 
-@pytest.mark.parametrize("variant", ["0", "1", "2", "3", "4", "5", "6", "7", "8", "9", "a", "b"])
+@pytest.mark.parametrize("variant", ["0", "1", "2", "3", "4", "5", "6", "7", "8", "9", "a", "b",
+                                     "i", "j", "m", "n", "w", "x"])
 def test_parity_3d_tile_variants(csx, monkeypatch, variant):
     """Every TC_TILE 3D CTA geometry / DMMA order (CSX_TILE3D_VARIANT), star and box, ragged
-    (y, x) tiles and z chunks, both boundaries."""
+    (y, x) tiles and z chunks, both boundaries (i / j / m / n / w / x: box-only variants — the
+    plane-interleaved order, two 8-warp CTAs per SM, 16-warp CTAs; stars take the default)."""
     monkeypatch.setenv("CSX_TILE3D_VARIANT", variant)
     for name, ext in (("heat3d", (70, 37, 45)), ("box3d27p", (9, 70, 150)), ("box3d27p", (37, 5, 9))):
         s = synth.SHAPES[name]
