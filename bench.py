@@ -630,9 +630,18 @@ def main():
             e1.record(stream)
             torch.cuda.synchronize()
             ems = e0.elapsed_time(e1) / e_steps
+            h_chunks, h2d_b, d2h_b = plan.host_last()
+            if h_chunks > 1:  # the C-ABI's ghost-zone chunk pipeline (include/csx.h csx_run_host)
+                dev = d_out.cpu().numpy()  # the device run's result (same input and T)
+                if np.max(np.abs(h_out - dev)) > 1e-12 * np.max(np.abs(dev)):
+                    raise SystemExit("chunked csx_run_host result differs from the device run")
+                how = (f"{h_chunks} ghost-zone chunks along the slowest axis, H2D(k+1) / run(k) / "
+                       "D2H(k-1) overlapped on three streams")
+            else:
+                how = "H2D + run + D2H serialised on one stream"
             sync_line = {"value": T * points / (ems * 1e-3) / 1e9, "unit": UNIT, "ms_per_step": ems,
-                         "api": "csx_run_host through the C-ABI (pinned host buffers; H2D + run + D2H "
-                                "serialised on one stream, timed by CUDA events)"}
+                         "api": f"csx_run_host through the C-ABI (pinned host buffers; {how}; timed by "
+                                "CUDA events around the calls)", "chunks": h_chunks}
             # A stream of grids through the same public calls: every step copies its own input
             # host->device and its whole result device->host, but step i+1's H2D and step i-1's
             # D2H (PCIe is full duplex) run on their own streams while step i computes.
@@ -673,7 +682,7 @@ def main():
             pms = e0.elapsed_time(e1) / K
             if not torch.equal(hout[(K - 1) % 2], ref.cpu()):
                 raise SystemExit("pipelined e2e result differs from the device run")
-            sync_line.update({"h2d_bytes_per_step": int(u0.nbytes), "d2h_bytes_per_step": int(u0.nbytes),
+            sync_line.update({"h2d_bytes_per_step": int(h2d_b), "d2h_bytes_per_step": int(d2h_b),
                               "steps": e_steps})
             sync_line["pipelined"] = {
                 "value": T * points / (pms * 1e-3) / 1e9, "unit": UNIT, "ms_per_step": pms,

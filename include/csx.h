@@ -123,9 +123,19 @@ csx_status csx_run(csx_plan_t plan, const double* d_in, double* d_out, int64_t t
 
 /* Same as csx_run, but d_in / d_out are HOST buffers (pageable or pinned): copies in, runs,
  * copies out, synchronises `stream` before returning.  The end-to-end call used by bench.py's
- * e2e leg. */
+ * e2e leg.  With pinned, distinct buffers and a grid of >= 8 (T + 1) r rows along its slowest
+ * axis, the call pipelines ghost-zone chunks of that axis (each chunk's rows plus (T + 1) r
+ * ghost rows per side, advanced by a sub-plan of the same stencil; the H2D copy of the next
+ * chunk, the run of this one and the D2H copy of the previous one overlap on three streams);
+ * results equal the whole-grid run up to rounding order.  Otherwise (pageable or in-place
+ * buffers, short grids, CSX_HOST_CHUNKS=0) one copy in, one run, one copy out.  The plan owns
+ * the chunk sub-plans and two device slots, freed by csx_plan_destroy.  h_in is never written. */
 csx_status csx_run_host(csx_plan_t plan, const double* h_in, double* h_out, int64_t timesteps,
                         void* stream);
+
+/* What the last csx_run_host on this plan did: chunks run (1 = serial path, 0 = none yet) and
+ * the bytes it copied host -> device (ghost rows included) and device -> host. */
+csx_status csx_host_last(const csx_plan_t plan, int* chunks, int64_t* h2d_bytes, int64_t* d2h_bytes);
 
 /* Multi-GPU (one process per GPU).  nccl_unique_id points to an ncclUniqueId
  * (NCCL_UNIQUE_ID_BYTES = 128 bytes) created by rank 0 and broadcast by the caller. */

@@ -84,6 +84,7 @@ _sig("csx_plan_lut", ctypes.c_int, [_vp, _i32p, _i32p, _i64p, ctypes.POINTER(cty
 
 _sig("csx_profile_enable", ctypes.c_int, [_vp, ctypes.c_int])
 _sig("csx_profile_read", ctypes.c_int, [_vp, ctypes.POINTER(ctypes.c_double), _i64p, _i64p, ctypes.c_int])
+_sig("csx_host_last", ctypes.c_int, [_vp, ctypes.POINTER(ctypes.c_int), _i64p, _i64p])
 
 _sig("csx_halo_schedule", ctypes.c_int, [_vp, ctypes.c_int, ctypes.c_int, _i64p, ctypes.POINTER(ctypes.c_int)])
 _sig("csx_plan_set_graph", ctypes.c_int, [_vp, ctypes.c_int])
@@ -94,7 +95,7 @@ _sig("csx_pencil_schedule", ctypes.c_int, [_vp, ctypes.c_int, ctypes.c_int, ctyp
 _sig("csx_run_sharded_pencil", ctypes.c_int, [_vp, _vp, ctypes.c_int, ctypes.c_int, _vp, _vp,
                                               ctypes.c_int64, _vp])
 
-EXPORTED = ["csx_plan_set_graph", "csx_plan_set_max_ctas", "csx_shard_box", "csx_pencil_schedule", "csx_run_sharded_pencil", "csx_peer_export", "csx_peer_connect", "csx_run_sharded_peer", "csx_auto_fuse_steps", "csx_plan_set_s2r_variant", "csx_halo_schedule", "csx_profile_enable", "csx_profile_read", "csx_plan", "csx_plan_set_engine", "csx_run", "csx_run_host", "csx_comm_create",
+EXPORTED = ["csx_host_last", "csx_plan_set_graph", "csx_plan_set_max_ctas", "csx_shard_box", "csx_pencil_schedule", "csx_run_sharded_pencil", "csx_peer_export", "csx_peer_connect", "csx_run_sharded_peer", "csx_auto_fuse_steps", "csx_plan_set_s2r_variant", "csx_halo_schedule", "csx_profile_enable", "csx_profile_read", "csx_plan", "csx_plan_set_engine", "csx_run", "csx_run_host", "csx_comm_create",
             "csx_comm_destroy", "csx_nccl_unique_id", "csx_shard_rows", "csx_run_sharded",
             "csx_plan_destroy", "csx_status_string", "csx_last_error", "csx_plan_info",
             "csx_compose_weights", "csx_weight_matrices", "csx_stencil2row_index",
@@ -244,6 +245,15 @@ def csx_profile_read(plan, reset: bool = True):
     return ms.value, tc.value, tot.value
 
 
+def csx_host_last(plan):
+    """(chunks, H2D bytes, D2H bytes) of the last csx_run_host on `plan`."""
+    k = ctypes.c_int()
+    hi = ctypes.c_int64()
+    ho = ctypes.c_int64()
+    _check(_lib.csx_host_last(plan, ctypes.byref(k), ctypes.byref(hi), ctypes.byref(ho)), "csx_host_last")
+    return k.value, hi.value, ho.value
+
+
 def csx_nccl_unique_id() -> bytes:
     buf = ctypes.create_string_buffer(128)
     _check(_lib.csx_nccl_unique_id(buf), "csx_nccl_unique_id")
@@ -377,6 +387,10 @@ class Plan:
             h_out = np.empty_like(h_in)
         csx_run_host(self._h, h_in, h_out, timesteps, stream)
         return h_out
+
+    def host_last(self):
+        """(chunks, H2D bytes, D2H bytes) of the last run_host."""
+        return csx_host_last(self._h)
 
     def shard_rows(self, rank: int, nranks: int):
         return csx_shard_rows(self._h, rank, nranks)

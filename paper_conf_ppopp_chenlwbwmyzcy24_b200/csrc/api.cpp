@@ -4,6 +4,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -510,12 +511,137 @@ csx_status csx_plan_set_graph(csx_plan_t p, int on) {
   return CSX_OK;
 }
 
+// csx_run_host, pipelined: the grid is cut along its slowest axis into K chunks; chunk k's
+// input is its rows plus a ghost zone of H = (T + 1) r rows on each side (wrapped for PERIODIC,
+// clipped at the global faces for FIXED), advanced T steps by a sub-plan of the same stencil,
+// boundary and fusion depth, and only its own rows are copied back.  Information travels r rows
+// per base step, and the sub-plan's artificial faces (held or wrapped) disturb at most the
+// T r + r rows next to them, so the kept rows equal the whole-grid run up to rounding order.  The
+// H2D copy of chunk k + 1, the run of chunk k and the D2H copy of chunk k - 1 overlap on three
+// streams (PCIe is full duplex), which hides most of the two copies behind the compute: 1 + 2H/C
+// of the work for two copies that took ~2/3 of the serial call.  Used when the host buffers are
+// pinned, distinct, and K >= 2 chunks of >= 4H rows exist (CSX_HOST_CHUNKS: 0 off, n forces n).
+static int host_chunks(const csx_plan_s* p, const double* h_in, double* h_out, int64_t T) {
+  const char* e = getenv("CSX_HOST_CHUNKS");
+  const int forced = e ? atoi(e) : -1;
+  if (forced == 0 || T <= 0 || h_in == h_out) return 0;
+  cudaPointerAttributes ai, ao;
+  if (cudaPointerGetAttributes(&ai, h_in) != cudaSuccess || cudaPointerGetAttributes(&ao, h_out) != cudaSuccess) {
+    cudaGetLastError();
+    return 0;
+  }
+  if (ai.type != cudaMemoryTypeHost || ao.type != cudaMemoryTypeHost) return 0;  // pageable: serial
+  const int64_t N = p->ext[0];
+  const int64_t H = (T + 1) * p->radius;
+  if (forced > 0) return (int)std::min<int64_t>(forced, std::max<int64_t>(1, N / (H + 1)));
+  const int64_t k = std::min<int64_t>(8, N / (4 * H));
+  return k >= 2 ? (int)k : 0;
+}
+
+static csx_status host_subplan(csx_plan_s* p, int64_t rows, csx_plan_s** out) {
+  for (auto& q : p->hsub)
+    if (q.first == rows) { *out = q.second; return CSX_OK; }
+  int64_t ext[3] = {p->ext[0], p->ext[1], p->ext[2]};
+  ext[0] = rows;
+  csx_plan_s* q = nullptr;
+  csx_status s = csx_plan(p->ndim, ext, p->shape, p->radius, p->w.data(), p->bc, p->tf, &q);
+  if (s != CSX_OK) return s;
+  s = csx_plan_set_engine(q, p->engine);
+  if (s == CSX_OK) s = csx_plan_set_max_ctas(q, p->max_ctas);
+  if (s != CSX_OK) { csx_plan_destroy(q); return s; }
+  p->hsub.emplace_back(rows, q);
+  *out = q;
+  return CSX_OK;
+}
+
+static csx_status run_host_chunked(csx_plan_s* p, const double* h_in, double* h_out, int64_t T,
+                                   cudaStream_t st, int K) {
+  const int64_t N = p->ext[0];
+  const int64_t plane = p->E[0] * p->E[1] * p->E[2] / N;  // doubles per slowest-axis row
+  const int64_t H = (T + 1) * p->radius;
+  const int64_t C = (N + K - 1) / K;
+  const bool per = p->bc == CSX_BC_PERIODIC;
+  const int64_t slot_rows = std::min<int64_t>(C + 2 * H, per ? C + 2 * H : N);
+  if (slot_rows * plane > p->h_slot_elems) {
+    for (auto& b : p->h_slot) { cudaFree(b); b = nullptr; }
+    p->h_slot_elems = 0;
+    for (auto& b : p->h_slot) {
+      cudaError_t e = cudaMalloc(&b, (size_t)(slot_rows * plane) * sizeof(double));
+      if (e != cudaSuccess) { cudaGetLastError(); return fail(CSX_ERR_OUT_OF_MEMORY, "cudaMalloc(host pipeline slot)"); }
+    }
+    p->h_slot_elems = slot_rows * plane;
+  }
+  if (!p->h_s_in) {
+    cudaStream_t a = nullptr, b = nullptr;
+    CSX_CUDA(cudaStreamCreateWithFlags(&a, cudaStreamNonBlocking), "stream");
+    p->h_s_in = a;
+    CSX_CUDA(cudaStreamCreateWithFlags(&b, cudaStreamNonBlocking), "stream");
+    p->h_s_out = b;
+    for (auto& ev : p->h_ev) {
+      cudaEvent_t x = nullptr;
+      CSX_CUDA(cudaEventCreateWithFlags(&x, cudaEventDisableTiming), "event");
+      ev = x;
+    }
+  }
+  cudaStream_t sin = (cudaStream_t)p->h_s_in, sout = (cudaStream_t)p->h_s_out;
+  cudaEvent_t* ev = reinterpret_cast<cudaEvent_t*>(p->h_ev);
+  // the caller's prior work on st (e.g. writes to h_in by an earlier D2H) precedes our copies
+  CSX_CUDA(cudaEventRecord(ev[2], st), "event");
+  CSX_CUDA(cudaStreamWaitEvent(sin, ev[2], 0), "wait");
+  const size_t rowb = (size_t)plane * sizeof(double);
+  p->h_last_chunks = 0;
+  p->h_last_h2d = p->h_last_d2h = 0;
+  for (int k = 0; k < K; ++k) {
+    const int64_t lo = k * C, hi = std::min(N, lo + C);
+    if (lo >= hi) break;
+    const int s = k & 1;
+    const int64_t r0 = per ? lo - H : std::max<int64_t>(0, lo - H);
+    const int64_t r1 = per ? hi + H : std::min(N, hi + H);
+    const int64_t rows = r1 - r0;
+    csx_plan_s* q = nullptr;
+    csx_status cs = host_subplan(p, rows, &q);
+    if (cs != CSX_OK) return cs;
+    double* din = p->h_slot[s];
+    double* dout = p->h_slot[2 + s];
+    // H2D of rows [r0, r1) (wrapped into [0, N) for PERIODIC: at most three runs)
+    if (k >= 2) CSX_CUDA(cudaStreamWaitEvent(sin, ev[2 + s], 0), "wait");  // chunk k-2's run done
+    for (int64_t r = r0; r < r1;) {
+      const int64_t g = ((r % N) + N) % N;
+      const int64_t len = std::min(r1 - r, N - g);
+      CSX_CUDA(cudaMemcpyAsync(din + (r - r0) * plane, h_in + g * plane, (size_t)len * rowb,
+                               cudaMemcpyHostToDevice, sin), "H2D");
+      r += len;
+    }
+    CSX_CUDA(cudaEventRecord(ev[s], sin), "event");
+    CSX_CUDA(cudaStreamWaitEvent(st, ev[s], 0), "wait");
+    if (k >= 2) CSX_CUDA(cudaStreamWaitEvent(st, ev[4 + s], 0), "wait");  // chunk k-2's D2H done
+    cs = csx_run(q, din, dout, T, st);
+    if (cs != CSX_OK) return cs;
+    CSX_CUDA(cudaEventRecord(ev[2 + s], st), "event");
+    CSX_CUDA(cudaStreamWaitEvent(sout, ev[2 + s], 0), "wait");
+    CSX_CUDA(cudaMemcpyAsync(h_out + lo * plane, dout + (lo - r0) * plane, (size_t)(hi - lo) * rowb,
+                             cudaMemcpyDeviceToHost, sout), "D2H");
+    CSX_CUDA(cudaEventRecord(ev[4 + s], sout), "event");
+    p->h_last_chunks += 1;
+    p->h_last_h2d += rows * (int64_t)rowb;
+    p->h_last_d2h += (hi - lo) * (int64_t)rowb;
+  }
+  CSX_CUDA(cudaStreamSynchronize(sout), "sync");
+  CSX_CUDA(cudaStreamSynchronize(st), "sync");
+  return CSX_OK;
+}
+
 csx_status csx_run_host(csx_plan_t p, const double* h_in, double* h_out, int64_t T, void* stream) {
   if (!p || !h_in || !h_out) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL argument");
+  if (T < 0) return fail(CSX_ERR_INVALID_ARGUMENT, "timesteps < 0");
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
   const int64_t n = p->E[0] * p->E[1] * p->E[2];
   csx_status s = ensure_device(p);
   if (s != CSX_OK) return s;
+  const int K = host_chunks(p, h_in, h_out, T);
+  if (K >= 2) return run_host_chunked(p, h_in, h_out, T, st, K);
+  p->h_last_chunks = 1;
+  p->h_last_h2d = p->h_last_d2h = n * (int64_t)sizeof(double);
   if (!p->d_dense) {
     cudaError_t e = cudaMalloc(&p->d_dense, n * sizeof(double));
     if (e != cudaSuccess) { cudaGetLastError(); return fail(CSX_ERR_OUT_OF_MEMORY, "cudaMalloc(dense)"); }
@@ -525,6 +651,14 @@ csx_status csx_run_host(csx_plan_t p, const double* h_in, double* h_out, int64_t
   if (s != CSX_OK) return s;
   CSX_CUDA(cudaMemcpyAsync(h_out, p->d_dense, n * sizeof(double), cudaMemcpyDeviceToHost, st), "D2H");
   CSX_CUDA(cudaStreamSynchronize(st), "sync");
+  return CSX_OK;
+}
+
+csx_status csx_host_last(const csx_plan_t p, int* chunks, int64_t* h2d_bytes, int64_t* d2h_bytes) {
+  if (!p) return fail(CSX_ERR_INVALID_ARGUMENT, "NULL plan");
+  if (chunks) *chunks = p->h_last_chunks;
+  if (h2d_bytes) *h2d_bytes = p->h_last_h2d;
+  if (d2h_bytes) *d2h_bytes = p->h_last_d2h;
   return CSX_OK;
 }
 
@@ -561,6 +695,8 @@ csx_status csx_profile_read(csx_plan_t p, double* tc_ms, int64_t* tc_launches, i
 
 csx_status csx_plan_destroy(csx_plan_t p) {
   if (!p) return CSX_OK;
+  for (auto& q : p->hsub) csx_plan_destroy(q.second);  // csx_run_host chunk sub-plans
+  p->hsub.clear();
   for (void* ev : p->prof_events) cudaEventDestroy((cudaEvent_t)ev);
   if (p->side) cudaStreamDestroy((cudaStream_t)p->side);
   if (p->ev_fork) cudaEventDestroy((cudaEvent_t)p->ev_fork);
@@ -579,6 +715,11 @@ csx_status csx_plan_destroy(csx_plan_t p) {
     cudaFree(p->d_buf[1]);
     cudaFree(p->d_wbase);
     cudaFree(p->d_dense);
+    for (auto& b : p->h_slot) cudaFree(b);
+    if (p->h_s_in) cudaStreamDestroy((cudaStream_t)p->h_s_in);
+    if (p->h_s_out) cudaStreamDestroy((cudaStream_t)p->h_s_out);
+    for (void* e : p->h_ev)
+      if (e) cudaEventDestroy((cudaEvent_t)e);
     if (!p->peer) {  // (peer plans keep their slab buffers inside the peer block)
       cudaFree(p->d_sbuf[0]);
       cudaFree(p->d_sbuf[1]);

@@ -4,6 +4,7 @@
 #pragma once
 #include <cstdint>
 #include <string>
+#include <utility>
 #include <vector>
 
 #include "../../include/csx.h"
@@ -141,6 +142,16 @@ struct csx_plan_s {
   double* d_pstage = nullptr;      // pencil halo staging (4 strided faces packed contiguously)
   size_t pstage_elems = 0;
   double* d_dense = nullptr;       // csx_run_host staging grid
+  // csx_run_host chunked pipeline (ghost-zone chunks along the slowest axis): sub-plans by
+  // chunk extent, two device slots (input / output), copy streams and per-slot events
+  std::vector<std::pair<int64_t, csx_plan_s*>> hsub;
+  double* h_slot[4] = {nullptr, nullptr, nullptr, nullptr};  // in0, in1, out0, out1
+  int64_t h_slot_elems = 0;
+  void* h_s_in = nullptr;          // cudaStream_t (H2D)
+  void* h_s_out = nullptr;         // cudaStream_t (D2H)
+  void* h_ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};  // h2d[2], comp[2], d2h[2]
+  int h_last_chunks = 0;           // what the last csx_run_host did (csx_host_last)
+  int64_t h_last_h2d = 0, h_last_d2h = 0;
   csx_peer_s* peer = nullptr;      // NVLink peer halo exchange (csx_peer_export / _connect)
   // side stream: the FIXED band fix-up of a TC_TILE 2D pass runs concurrently with the pass
   void* side = nullptr;            // cudaStream_t

@@ -1772,6 +1772,7 @@ using Tile3D7ks = Tile3DCfg<7, 4, 2, 4, 10, 32, 1, 1, 4, 2, 0, 4>;
 using Tile3D5w = Tile3DCfg<5, 4, 8, 2, 6, 32, 1, 1, 2, 4, 0, 0, 1>;
 using Tile3D7w = Tile3DCfg<7, 2, 4, 4, 10, 32, 1, 1, 4, 2, 0, 4>;
 using Tile3D3w16 = Tile3DCfg<3, 4, 4, 4, 6, 32, 1, 1>;
+using Tile3D7w1 = Tile3DCfg<7, 1, 4, 4, 10, 32, 1, 1, 4, 2, 0, 4>;  // star r = 3: 16 warps of one block row, CTA 16 x 64
 using Tile3D3w16r = Tile3DCfg<3, 4, 4, 4, 6, 32, 1, 0>;  // row-outer DMMA order (boxes)
 using Tile3D5w16 = Tile3DCfg<5, 2, 8, 2, 9, 32, 1, 1, 2, 4, 0>;  // box r = 2, 16 warps, CTA 32 x 64
 using Tile3D7w16 = Tile3DCfg<7, 2, 4, 4, 10, 32, 1, 1, 4, 2, 0>;  // box r = 3, 16 warps, CTA 32 x 64
@@ -2141,6 +2142,7 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
       // GSt/s); r = 3 stars spill at 16 warps (121.7 -> 96.4) and keep 8 unless W16 = 1
       const char* w16 = getenv("CSX_TILE3D_W16");
       const bool w16_on = w16 ? w16[0] == '1' : nk == 5;
+      if (star && scf && nk == 7 && w16 && w16[0] == '2') return launch_tile3d_cfg<Tile3D7w1>(a, a.tc_mask, st);
       if (star && scf && w16_on)
         return nk == 5 ? launch_tile3d_cfg<Tile3D5w>(a, a.tc_mask, st) : launch_tile3d_cfg<Tile3D7w>(a, a.tc_mask, st);
       if (nk == 5 && (g8 ? g8[0] == '1' : star))

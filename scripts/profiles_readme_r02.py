@@ -103,14 +103,14 @@ if os.path.exists(lc):
 
 out = f"""# Round 2 profiles (B200, sm_100a)
 
-Measured at HEAD through gpurun (`scripts/r02_full2.sh`): the whole GPU suite (`gpu_all.log`),
+Measured at HEAD through gpurun (`scripts/r02_final2.sh`; earlier passes `r02_full2.sh`, `r02_final.sh`): the whole GPU suite (`gpu_all.log`),
 `smoke()` (`smoke.log`), one bench line per config (`bench_all.jsonl`: TC_TILE / auto engine with
 the CUDA-core comparator at its own fusion depth, e2e through `csx_run_host`, the ncu counters
 of the committed DMMA pass), the paper's layout (`bench_s2r.jsonl`), the plain `python bench.py`
 line (`bench_default.json`), the reference arm (`bench_reference.json`: the oracle on the
 host cores), the DMMA / FP64-pipe / DRAM counters of every dominant kernel
 (`dmma_counters.json`, `scripts/dmma_counters.py`), `ncu --set full` briefs of the round-2
-kernels (`brief/`), sanitizers (`*check*.txt`) and the launch list of the default bench.  ncu
+kernels with their SASS stall maps (`brief/`), sanitizers of earlier passes (`*check*.txt`) and the launch list of the default bench.  ncu
 runs are cold-cache and serialised: compare shares and counters, not absolute times.
 This file's tables are regenerated by `scripts/profiles_readme_r02.py`.
 

@@ -721,3 +721,31 @@ def test_tile1d_variants(variant):
                          capture_output=True, text=True, timeout=300)
     assert out.returncode == 0, out.stderr[-2000:]
     assert float(out.stdout.strip().splitlines()[-1]) <= TOL, (variant, out.stdout)
+
+
+@pytest.mark.parametrize("name, ext, T", [
+    ("heat1d", (40001,), 23), ("1d5p", (30001,), 11), ("box2d9p", (301, 130), 7), ("heat2d", (257, 96), 10),
+    ("box2d49p", (200, 70), 3), ("heat3d", (70, 33, 40), 5), ("box3d27p", (61, 20, 36), 3)])
+@pytest.mark.parametrize("bc", ["fixed", "periodic"])
+def test_run_host_chunked_pipeline(csx, monkeypatch, name, ext, T, bc):
+    """csx_run_host with pinned host buffers runs ghost-zone chunks along the slowest axis on
+    three streams (H2D of chunk k+1 / run of chunk k / D2H of chunk k-1): forced to 2, 3 and 5
+    chunks (CSX_HOST_CHUNKS) — chunks whose ghost zones wrap (PERIODIC) or clip at the global
+    faces (FIXED), a short last chunk — and compared element by element with the oracle; pageable
+    buffers and CSX_HOST_CHUNKS = 0 take the serial path."""
+    s = synth.SHAPES[name]
+    w = synth.random_weights(name)
+    u0 = synth.grid(ext, seed=77)
+    ref = oracle.run(u0, w, bc, T)
+    p = csx.Plan(u0.shape, w, shape=s.kind, bc=bc)
+    h_in = torch.from_numpy(u0).pin_memory().numpy()
+    for k in ("2", "3", "5", "0"):
+        monkeypatch.setenv("CSX_HOST_CHUNKS", k)
+        h_out = torch.empty(u0.shape, dtype=torch.float64).pin_memory().numpy()
+        h_out[...] = np.nan
+        p.run_host(h_in, T, h_out)
+        assert rel(h_out, ref) <= TOL, (name, bc, k)
+    monkeypatch.delenv("CSX_HOST_CHUNKS")
+    got = p.run_host(u0.copy(), T)            # pageable: serial path
+    assert rel(got, ref) <= TOL
+    p.close()
