@@ -524,7 +524,13 @@ csx_status csx_plan_set_graph(csx_plan_t p, int on) {
 static int host_chunks(const csx_plan_s* p, const double* h_in, double* h_out, int64_t T) {
   const char* e = getenv("CSX_HOST_CHUNKS");
   const int forced = e ? atoi(e) : -1;
-  if (forced == 0 || T <= 0 || h_in == h_out) return 0;
+  if (forced == 0 || T <= 0) return 0;
+  {  // overlapping host buffers (in place or not): the serial path reads all input first
+    const int64_t n = p->E[0] * p->E[1] * p->E[2];
+    const uintptr_t a0 = reinterpret_cast<uintptr_t>(h_in), a1 = a0 + (uintptr_t)n * sizeof(double);
+    const uintptr_t b0 = reinterpret_cast<uintptr_t>(h_out), b1 = b0 + (uintptr_t)n * sizeof(double);
+    if (a0 < b1 && b0 < a1) return 0;
+  }
   cudaPointerAttributes ai, ao;
   if (cudaPointerGetAttributes(&ai, h_in) != cudaSuccess || cudaPointerGetAttributes(&ao, h_out) != cudaSuccess) {
     cudaGetLastError();
@@ -589,6 +595,16 @@ static csx_status run_host_chunked(csx_plan_s* p, const double* h_in, double* h_
   CSX_CUDA(cudaEventRecord(ev[2], st), "event");
   CSX_CUDA(cudaStreamWaitEvent(sin, ev[2], 0), "wait");
   const size_t rowb = (size_t)plane * sizeof(double);
+  // every chunk's sub-plan first: a chunk shorter than its composed window (tiny grids, few
+  // steps, deep fusion) is refused by csx_plan, and then the whole call takes the serial path
+  for (int k = 0; k < K; ++k) {
+    const int64_t lo = k * C, hi = std::min(N, lo + C);
+    if (lo >= hi) break;
+    const int64_t r0 = per ? lo - H : std::max<int64_t>(0, lo - H);
+    const int64_t r1 = per ? hi + H : std::min(N, hi + H);
+    csx_plan_s* q = nullptr;
+    if (host_subplan(p, r1 - r0, &q) != CSX_OK) return CSX_ERR_UNSUPPORTED;
+  }
   p->h_last_chunks = 0;
   p->h_last_h2d = p->h_last_d2h = 0;
   for (int k = 0; k < K; ++k) {
@@ -639,7 +655,11 @@ csx_status csx_run_host(csx_plan_t p, const double* h_in, double* h_out, int64_t
   csx_status s = ensure_device(p);
   if (s != CSX_OK) return s;
   const int K = host_chunks(p, h_in, h_out, T);
-  if (K >= 2) return run_host_chunked(p, h_in, h_out, T, st, K);
+  if (K >= 2) {
+    s = run_host_chunked(p, h_in, h_out, T, st, K);
+    if (s != CSX_ERR_UNSUPPORTED) return s;
+    set_error("");  // a chunk too short for its sub-plan: serial path below
+  }
   p->h_last_chunks = 1;
   p->h_last_h2d = p->h_last_d2h = n * (int64_t)sizeof(double);
   if (!p->d_dense) {

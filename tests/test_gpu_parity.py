@@ -749,3 +749,31 @@ def test_run_host_chunked_pipeline(csx, monkeypatch, name, ext, T, bc):
     got = p.run_host(u0.copy(), T)            # pageable: serial path
     assert rel(got, ref) <= TOL
     p.close()
+
+
+def test_run_host_chunks_fall_back(csx, monkeypatch):
+    """Forced chunks too short for the fused window (nk = 27 sub-plans on 12-row chunks) and
+    overlapping host buffers take the serial path; results stay equal to the oracle."""
+    w = synth.random_weights("heat1d")
+    u0 = synth.grid((60,), seed=5)
+    ref = oracle.run(u0, w, "fixed", 15)
+    p = csx.Plan(u0.shape, w, shape="star", bc="fixed", fuse_steps=13)
+    monkeypatch.setenv("CSX_HOST_CHUNKS", "5")
+    h_in = torch.from_numpy(u0).pin_memory().numpy()
+    h_out = torch.empty(u0.shape, dtype=torch.float64).pin_memory().numpy()
+    p.run_host(h_in, 15, h_out)
+    assert rel(h_out, ref) <= TOL
+    assert p.host_last()[0] == 1
+    p.close()
+    w2 = synth.random_weights("box2d9p")
+    u2 = synth.grid((300, 64), seed=6)
+    ref2 = oracle.run(u2, w2, "periodic", 7)
+    p2 = csx.Plan(u2.shape, w2, shape="box", bc="periodic")
+    big = torch.from_numpy(np.concatenate([u2.ravel(), np.zeros(64)])).pin_memory().numpy()
+    src = big[:u2.size].reshape(u2.shape)
+    dst = big[64:64 + u2.size].reshape(u2.shape)       # overlaps src, shifted by one row
+    monkeypatch.setenv("CSX_HOST_CHUNKS", "3")
+    p2.run_host(src, 7, dst)
+    assert p2.host_last()[0] == 1
+    assert rel(dst, ref2) <= TOL
+    p2.close()
