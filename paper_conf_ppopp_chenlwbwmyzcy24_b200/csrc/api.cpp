@@ -520,7 +520,8 @@ csx_status csx_plan_set_graph(csx_plan_t p, int on) {
 // H2D copy of chunk k + 1, the run of chunk k and the D2H copy of chunk k - 1 overlap on three
 // streams (PCIe is full duplex), which hides most of the two copies behind the compute: 1 + 2H/C
 // of the work for two copies that took ~2/3 of the serial call.  Used when the host buffers are
-// pinned, distinct, and K >= 2 chunks of >= 4H rows exist (CSX_HOST_CHUNKS: 0 off, n forces n).
+// pinned and do not overlap, and K >= 2 chunks of >= 4H rows and >= 8M points exist (K <= 4;
+// CSX_HOST_CHUNKS: 0 off, n forces n).
 static int host_chunks(const csx_plan_s* p, const double* h_in, double* h_out, int64_t T) {
   const char* e = getenv("CSX_HOST_CHUNKS");
   const int forced = e ? atoi(e) : -1;
@@ -540,7 +541,13 @@ static int host_chunks(const csx_plan_s* p, const double* h_in, double* h_out, i
   const int64_t N = p->ext[0];
   const int64_t H = (T + 1) * p->radius;
   if (forced > 0) return (int)std::min<int64_t>(forced, std::max<int64_t>(1, N / (H + 1)));
-  const int64_t k = std::min<int64_t>(8, N / (4 * H));
+  // up to 4 chunks of >= 4H rows (ghost rows <= 50 % of a chunk) and >= 8M points each (so each
+  // chunk's passes stay long kernels, not launch-bound): measured on C2, 4 chunks 367 GSt/s,
+  // 8: 332, 12: 310, 16: 285 (serial 220); 8 chunks of the 10.24M-point 1D grid ran slower
+  // than the serial call (their 77 passes of 1.3M points each are launch-bound)
+  const int64_t plane = p->E[0] * p->E[1] * p->E[2] / N;
+  int64_t k = std::min<int64_t>(4, N / (4 * H));
+  while (k >= 2 && (N / k) * plane < (int64_t(8) << 20)) --k;
   return k >= 2 ? (int)k : 0;
 }
 
