@@ -327,8 +327,8 @@ csx_status build_pass(const csx_plan_s* p, int tf, Pass* out) {
 }
 
 int auto_tf(int ndim, int radius, int engine) {
-  // DESIGN.md "Fusion depth" (reading A4): 2D r=1 -> 3 (the paper's Box-2D9P choice,
-  // P.1478-1480); r >= 2 in 2D and all 3D -> 1 (one N fragment, lowest DMMA count per
+  // DESIGN.md "Fusion depth" (reading A4): 2D r=1 -> 2 (TC_TILE on B200; TC_S2R keeps the
+  // paper's Box-2D9P choice of 3, P.1478-1480); r >= 2 in 2D and all 3D -> 1 (one N fragment, lowest DMMA count per
   // point-step on B200).  1D is HBM-bound, so deeper fusion pays until the DMMA work of the
   // Toeplitz blocks (K = nk + 7) meets the HBM time: TC_TILE takes nk ~ 27..29 (r=1 -> 13,
   // r=2 -> 7, r=3 -> 3; round-2 sweep on Heat-1D / 1D5P, 10.24M and 102.4M points: Tf 9 / 11 /
@@ -342,7 +342,13 @@ int auto_tf(int ndim, int radius, int engine) {
   // the CUDA-core comparator's own best depth: 2D r = 1 -> 4 (register wavefront, Box-2D9P
   // 10240^2: Tf 1/2/3/4 = 310 / 640 / 681 / 766 GSt/s), r >= 2 -> 1
   if (ndim == 2 && engine == CSX_ENGINE_DIRECT) return radius == 1 ? 4 : 1;
-  if (ndim == 2) return radius == 1 ? 3 : 1;
+  // 2D r = 1: the paper fuses 3 steps (Box-2D9P, P.1478-1480) and so does its layout here
+  // (TC_S2R: 26 DMMAs per 64 outputs at nk = 7 vs 14 per 48 at nk = 5).  TC_TILE on B200 runs 2:
+  // nk = 5 executes 48 tensor flops per point-step against nk = 7's 53.3 and moves 8 B instead
+  // of 5.3, which the 6.5 TB/s HBM still covers — Box-2D9P / Heat-2D 10240^2, T = 100: 640 /
+  // 640 GSt/s at Tf = 2 against 618 / 618 at Tf = 3 and 510 at Tf = 4 (profiles/r02/ab/)
+  if (ndim == 2 && engine == CSX_ENGINE_TC_S2R) return radius == 1 ? 3 : 1;
+  if (ndim == 2) return radius == 1 ? 2 : 1;
   return 1;
 }
 

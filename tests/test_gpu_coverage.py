@@ -140,7 +140,7 @@ def test_persistent_ctas_wrap(csx, case, bc):
 FULL = [
     # (name, extents, T, fuse_steps list): BASELINE.json configs C1-C4 plus the north-star 1D list
     ("heat1d", (1024,), 16, [0]),                       # C1
-    ("box2d9p", (10240, 10240), 100, [0]),              # C2 (the headline; auto Tf = 3)
+    ("box2d9p", (10240, 10240), 100, [0, 3]),           # C2 (the headline; auto Tf = 2, and the paper's 3)
     ("star2d13p", (10240, 10240), 100, [0, 2]),         # C3, auto (Tf = 1) and "multi-step fused"
     ("box2d49p", (10240, 10240), 100, [0, 2]),          # C3
     ("heat3d", (512, 512, 512), 50, [0]),               # C4

@@ -258,7 +258,7 @@ def test_2d_fusion_limits():
 
 def test_auto_fusion_depths():
     # (3D r = 1 stars run two steps per pass by temporal blocking; boxes and r >= 2 one)
-    cases = {"heat1d": 13, "1d5p": 7, "heat2d": 3, "box2d9p": 3, "star2d13p": 1, "box2d49p": 1,
+    cases = {"heat1d": 13, "1d5p": 7, "heat2d": 2, "box2d9p": 2, "star2d13p": 1, "box2d49p": 1,
              "heat3d": 2, "box3d27p": 1, "star3d13p": 1, "box3d125p": 1}
     for name, tf in cases.items():
         s = synth.SHAPES[name]
@@ -271,6 +271,10 @@ def test_auto_fusion_depths():
         p = csx.Plan((4096,), synth.physical_weights(name), engine="tc_s2r")
         assert p.info()["fuse_steps"] == tf and p.info()["engine_name"] == "tc_s2r", name
         p.close()
+    # 2D r = 1: TC_TILE fuses 2 steps on B200, the paper's layout (TC_S2R) keeps its 3
+    p = csx.Plan((128, 128), synth.physical_weights("box2d9p"), engine="tc_s2r")
+    assert p.info()["fuse_steps"] == 3 and p.info()["nk"] == 7
+    p.close()
     assert csx._lib.csx_auto_fuse_steps(1, 3, csx.ENGINES["tc_tile"]) == 3
     # the CUDA-core comparator's own depth (2D r = 1: 4 steps)
     assert csx._lib.csx_auto_fuse_steps(2, 1, csx.ENGINES["direct"]) == 4
