@@ -545,8 +545,11 @@ static int host_chunks(const csx_plan_s* p, const double* h_in, double* h_out, i
   // chunk's passes stay long kernels, not launch-bound): measured on C2, 4 chunks 367 GSt/s,
   // 8: 332, 12: 310, 16: 285 (serial 220); 8 chunks of the 10.24M-point 1D grid ran slower
   // than the serial call (their 77 passes of 1.3M points each are launch-bound)
+  // Where the ghost rows are cheap (<= 10 % of the grid over all chunks) up to 8 chunks: the
+  // 102.4M-point 1D grid ran 3597 GSt/s with 8 chunks, 3236 with 4.
   const int64_t plane = p->E[0] * p->E[1] * p->E[2] / N;
-  int64_t k = std::min<int64_t>(4, N / (4 * H));
+  int64_t k = std::min<int64_t>(8, (N / 10) / (2 * H));
+  if (k < 2) k = std::min<int64_t>(4, N / (4 * H));
   while (k >= 2 && (N / k) * plane < (int64_t(8) << 20)) --k;
   return k >= 2 ? (int)k : 0;
 }
