@@ -124,7 +124,7 @@ csx_status csx_run(csx_plan_t plan, const double* d_in, double* d_out, int64_t t
 /* Same as csx_run, but d_in / d_out are HOST buffers (pageable or pinned): copies in, runs,
  * copies out, synchronises `stream` before returning.  The end-to-end call used by bench.py's
  * e2e leg.  With pinned, non-overlapping buffers and a grid of >= 8 (T + 1) r rows and >= 16M
- * points, the call pipelines up to 4 ghost-zone chunks of its slowest axis (each chunk's rows plus (T + 1) r
+ * points, the call pipelines up to 8 ghost-zone chunks of its slowest axis (each chunk's rows plus (T + 1) r
  * ghost rows per side, advanced by a sub-plan of the same stencil; the H2D copy of the next
  * chunk, the run of this one and the D2H copy of the previous one overlap on three streams);
  * results equal the whole-grid run up to rounding order.  Otherwise (pageable or overlapping
