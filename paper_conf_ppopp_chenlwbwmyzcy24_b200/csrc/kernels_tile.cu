@@ -1772,6 +1772,8 @@ using Tile3D7ks = Tile3DCfg<7, 4, 2, 4, 10, 32, 1, 1, 4, 2, 0, 4>;
 using Tile3D5w = Tile3DCfg<5, 4, 8, 2, 6, 32, 1, 1, 2, 4, 0, 0, 1>;
 using Tile3D7w = Tile3DCfg<7, 2, 4, 4, 10, 32, 1, 1, 4, 2, 0, 4>;
 using Tile3D3w16 = Tile3DCfg<3, 4, 4, 4, 6, 32, 1, 1>;
+using Tile3D3z16 = Tile3DCfg<3, 4, 2, 8, 6, 32, 1, 1>;   // r = 1: 16 warps, CTA 32 x 128 (x halo 4 / 128)
+using Tile3D3u = Tile3DCfg<3, 8, 1, 8, 6, 32, 1, 1>;     // r = 1: 8 warps, CTA 32 x 128
 using Tile3D7w1 = Tile3DCfg<7, 1, 4, 4, 10, 32, 1, 1, 4, 2, 0, 4>;  // star r = 3: 16 warps of one block row, CTA 16 x 64
 using Tile3D3w16r = Tile3DCfg<3, 4, 4, 4, 6, 32, 1, 0>;  // row-outer DMMA order (boxes)
 using Tile3D5w16 = Tile3DCfg<5, 2, 8, 2, 9, 32, 1, 1, 2, 4, 0>;  // box r = 2, 16 warps, CTA 32 x 64
@@ -2169,6 +2171,8 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
       if (e && e[0] == '7') return launch_tile3d_cfg<Tile3D3l>(a, a.tc_mask, st);
       if (e && e[0] == 'a') return launch_tile3d_cfg<Tile3D3za>(a, a.tc_mask, st);
       if (e && e[0] == 'b') return launch_tile3d_cfg<Tile3D3zb>(a, a.tc_mask, st);
+      if (e && e[0] == 'z') return launch_tile3d_cfg<Tile3D3z16>(a, a.tc_mask, st);
+      if (e && e[0] == 'u') return launch_tile3d_cfg<Tile3D3u>(a, a.tc_mask, st);
       // default: star shapes (one TC plane, HBM-bound) take the 64 x 64 tile with 8 DMMA warps
       // (less halo per plane); box shapes (DMMA-bound) the 64 x 32 tile at 2 CTAs / SM
       // (measured)

@@ -287,11 +287,12 @@ def test_parity_3d_two_step_blocking(csx, name, bc):
 
 
 @pytest.mark.parametrize("variant", ["0", "1", "2", "3", "4", "5", "6", "7", "8", "9", "a", "b",
-                                     "i", "j", "m", "n", "w", "x"])
+                                     "i", "j", "m", "n", "w", "x", "z", "u"])
 def test_parity_3d_tile_variants(csx, monkeypatch, variant):
     """Every TC_TILE 3D CTA geometry / DMMA order (CSX_TILE3D_VARIANT), star and box, ragged
     (y, x) tiles and z chunks, both boundaries (i / j / m / n / w / x: box-only variants — the
-    plane-interleaved order, two 8-warp CTAs per SM, 16-warp CTAs; stars take the default)."""
+    plane-interleaved order, two 8-warp CTAs per SM, 16-warp CTAs; z / u: 32 x 128 tiles of 16 /
+    8 warps; stars take the default unless noted)."""
     monkeypatch.setenv("CSX_TILE3D_VARIANT", variant)
     for name, ext in (("heat3d", (70, 37, 45)), ("box3d27p", (9, 70, 150)), ("box3d27p", (37, 5, 9))):
         s = synth.SHAPES[name]
