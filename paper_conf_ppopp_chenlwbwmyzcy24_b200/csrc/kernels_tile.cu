@@ -1172,6 +1172,8 @@ static cudaError_t launch_tile3d_tb(S2RArgs a, int tc_mask, cudaStream_t st) {
 template <int IN_ = 4, int L1S_ = 5, int WIDE_ = 1, int BM_ = 32, int BAL_ = 0>
 struct Tile3DTB2 {
   static constexpr int BAL = BAL_;
+  // BM = 16: two CTAs per SM (two independent level-1 / level-2 pipelines per SM)
+  static constexpr int MINB = BM_ <= 16 ? 2 : 1;
   static constexpr int R = 1, A = 4, B = 2, KR = 6, KS = 6, H = 2, ZCH = 32;
   // WIDE = 1: 32 x 64 output tile, step-1 plane 36 x 80 (level-1 warps: 5 DMMA tiles each),
   //           inputs of output (row, col) at staged (row + dy, col + 1 + dx)   [OFF = 1]
@@ -1235,7 +1237,7 @@ __device__ __forceinline__ void tb_hwindow(double (&acc)[G][2], const double* co
 }
 
 template <bool ONE, class D>  // ONE: a single TC plane (star shapes): only its fragments in registers
-__global__ void __launch_bounds__(D::NT, 1)
+__global__ void __launch_bounds__(D::NT, D::MINB)
     k_tile3d_tb2(S2RArgs a, int tc_mask, const __grid_constant__ CUtensorMap tmap) {
   extern __shared__ __align__(128) double smem_raw[];
   double* smem = ring_base(smem_raw);
@@ -2016,11 +2018,12 @@ static cudaError_t launch_tile1d(int nk, const S2RArgs& a, cudaStream_t st) {
 
 // 3D Tf = 2 geometry (CSX_TB_GEOM, read per call; the planner's DMMA count follows the same
 // choice): '0' tb2 32 x 62, '1' tb2 32 x 64 roles by warp index, 't' tb2 32 x 64 balanced roles,
-// '3'-'5' tb2 28 x 64, '6' / '8' tb2 ring depths, 'a'-'c' tb3 strip tiles
+// '3'-'5' tb2 28 x 64, '6' / '8' tb2 ring depths, 'a'-'c' tb3 strip tiles, 'h' tb2 16 x 64 at two
+// CTAs per SM
 #define CSX_TB_GEOM_DEFAULT 't'
 static char tb_geom() {
   const char* r = getenv("CSX_TB_GEOM");
-  if (r && r[0] && std::strchr("0134568abct", r[0])) return r[0];
+  if (r && r[0] && std::strchr("0134568abcht", r[0])) return r[0];
   return CSX_TB_GEOM_DEFAULT;  // balanced roles (Heat-3D 315.0 -> 320.0 GSt/s)
 }
 
@@ -2032,6 +2035,7 @@ double tile3d_tb_mma_per_point() {
     case '0': return (36.0 * 34.0 / 32.0 + 32.0) * 6.0 / (32.0 * 62.0);  // step-1 36 x 64
     case '3': case '4': case '5': return (40.0 * 34.0 / 32.0 + 28.0) * 6.0 / (28.0 * 64.0);
     case 'a': case 'b': case 'c': return (39.0 * 34.0 / 32.0 + 32.0) * 6.0 / (32.0 * 64.0);
+    case 'h': return (25.0 * 34.0 / 32.0 + 16.0) * 6.0 / (16.0 * 64.0);  // step-1 20 x 80
     default: return (45.0 * 34.0 / 32.0 + 32.0) * 6.0 / (32.0 * 64.0);  // step-1 36 x 80
   }
 }
@@ -2124,6 +2128,7 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
       // (BM = 28, geometries 3-5: 16 warps, balanced sub-partitions, deeper rings: 281-296 GSt/s, slower)
       if (r && r[0] == '1') return launch_tile3d_tb2<Tile3DTB2<4, 5, 1>>(a, a.tc_mask, st);  // unbalanced roles
       if (r && r[0] == 't') return launch_tile3d_tb2<Tile3DTB2<4, 5, 1, 32, 1>>(a, a.tc_mask, st);
+      if (r && r[0] == 'h') return launch_tile3d_tb2<Tile3DTB2<4, 4, 1, 16>>(a, a.tc_mask, st);
       if (r && r[0] == 'a') return launch_tile3d_tb3<Tile3DTB3<5, 5>>(a, a.tc_mask, st);
       if (r && r[0] == 'b') return launch_tile3d_tb3<Tile3DTB3<4, 6>>(a, a.tc_mask, st);
       if (r && r[0] == 'c') return launch_tile3d_tb3<Tile3DTB3<6, 4>>(a, a.tc_mask, st);

@@ -301,7 +301,7 @@ def test_randomized_plans_against_oracle(csx):
     assert ran >= 120, ran
 
 
-@pytest.mark.parametrize("geom", ["0", "1", "3", "4", "5", "6", "8", "a", "b", "c", "t"])
+@pytest.mark.parametrize("geom", ["0", "1", "3", "4", "5", "6", "8", "a", "b", "c", "h", "t"])
 def test_tb2_geometries(csx, monkeypatch, geom):
     """Every k_tile3d_tb2 / k_tile3d_tb3 geometry (CSX_TB_GEOM; a-c: tb3's strip tiles with three
     ring depths, t: the balanced-role tb2 32 x 64 tile):

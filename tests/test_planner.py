@@ -341,7 +341,7 @@ def test_status_strings():
 
 @pytest.mark.parametrize("geom, l1_tiles, rows, cols", [
     (None, 45, 32, 64), ("t", 45, 32, 64), ("1", 45, 32, 64), ("a", 39, 32, 64), ("c", 39, 32, 64),
-    ("3", 40, 28, 64), ("0", 36, 32, 62)])
+    ("3", 40, 28, 64), ("0", 36, 32, 62), ("h", 25, 16, 64)])
 def test_3d_two_step_mma_count(monkeypatch, geom, l1_tiles, rows, cols):
     """3D Tf = 2 (temporal blocking of the base r = 1 window): the planner's DMMA count per pass
     follows the geometry CSX_TB_GEOM selects — (level-1 DMMA tiles x 34/32 planes + level-2
