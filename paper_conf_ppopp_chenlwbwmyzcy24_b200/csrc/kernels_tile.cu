@@ -2118,21 +2118,20 @@ cudaError_t launch_tile(int ndim, int radius, int tf, const S2RArgs& a, cudaStre
     if (tf == 2) {  // r = 1: temporal blocking (CSX_TB=1: the round-1 single-barrier kernel)
       const char* e = getenv("CSX_TB");
       if (e && e[0] == '1') return launch_tile3d_tb<Tile3DTB>(a, a.tc_mask, st);
-      const char g = tb_geom();
-      const char* r = &g;  // 0: the 32 x 62 tile (equal level work)
-      if (r && r[0] == '0') return launch_tile3d_tb2<Tile3DTB2<5, 6, 0>>(a, a.tc_mask, st);
-      if (r && r[0] == '3') return launch_tile3d_tb2<Tile3DTB2<5, 5, 1, 28>>(a, a.tc_mask, st);
-      if (r && r[0] == '4') return launch_tile3d_tb2<Tile3DTB2<4, 6, 1, 28>>(a, a.tc_mask, st);
-      if (r && r[0] == '5') return launch_tile3d_tb2<Tile3DTB2<6, 4, 1, 28>>(a, a.tc_mask, st);
-      if (r && r[0] == '6') return launch_tile3d_tb2<Tile3DTB2<5, 4, 1, 32>>(a, a.tc_mask, st);
+      const char g = tb_geom();  // 0: the 32 x 62 tile (equal level work), ... (see tb_geom)
+      if (g == '0') return launch_tile3d_tb2<Tile3DTB2<5, 6, 0>>(a, a.tc_mask, st);
+      if (g == '3') return launch_tile3d_tb2<Tile3DTB2<5, 5, 1, 28>>(a, a.tc_mask, st);
+      if (g == '4') return launch_tile3d_tb2<Tile3DTB2<4, 6, 1, 28>>(a, a.tc_mask, st);
+      if (g == '5') return launch_tile3d_tb2<Tile3DTB2<6, 4, 1, 28>>(a, a.tc_mask, st);
+      if (g == '6') return launch_tile3d_tb2<Tile3DTB2<5, 4, 1, 32>>(a, a.tc_mask, st);
       // (BM = 28, geometries 3-5: 16 warps, balanced sub-partitions, deeper rings: 281-296 GSt/s, slower)
-      if (r && r[0] == '1') return launch_tile3d_tb2<Tile3DTB2<4, 5, 1>>(a, a.tc_mask, st);  // unbalanced roles
-      if (r && r[0] == 't') return launch_tile3d_tb2<Tile3DTB2<4, 5, 1, 32, 1>>(a, a.tc_mask, st);
-      if (r && r[0] == 'h') return launch_tile3d_tb2<Tile3DTB2<4, 4, 1, 16>>(a, a.tc_mask, st);
-      if (r && r[0] == 'a') return launch_tile3d_tb3<Tile3DTB3<5, 5>>(a, a.tc_mask, st);
-      if (r && r[0] == 'b') return launch_tile3d_tb3<Tile3DTB3<4, 6>>(a, a.tc_mask, st);
-      if (r && r[0] == 'c') return launch_tile3d_tb3<Tile3DTB3<6, 4>>(a, a.tc_mask, st);
-      if (r && r[0] == '8') return launch_tile3d_tb2<Tile3DTB2<5, 4, 1, 32, 1>>(a, a.tc_mask, st);
+      if (g == '1') return launch_tile3d_tb2<Tile3DTB2<4, 5, 1>>(a, a.tc_mask, st);  // unbalanced roles
+      if (g == 't') return launch_tile3d_tb2<Tile3DTB2<4, 5, 1, 32, 1>>(a, a.tc_mask, st);
+      if (g == 'h') return launch_tile3d_tb2<Tile3DTB2<4, 4, 1, 16>>(a, a.tc_mask, st);
+      if (g == 'a') return launch_tile3d_tb3<Tile3DTB3<5, 5>>(a, a.tc_mask, st);
+      if (g == 'b') return launch_tile3d_tb3<Tile3DTB3<4, 6>>(a, a.tc_mask, st);
+      if (g == 'c') return launch_tile3d_tb3<Tile3DTB3<6, 4>>(a, a.tc_mask, st);
+      if (g == '8') return launch_tile3d_tb2<Tile3DTB2<5, 4, 1, 32, 1>>(a, a.tc_mask, st);
       return cudaErrorNotSupported;
     }
     if (nk == 5 || nk == 7) {
